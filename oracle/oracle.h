@@ -1,0 +1,85 @@
+/*
+ * oracle.h -- plain, slow, obviously-correct CPU oracle for the Paraprox
+ * Stencil & Partition approximation (Samadi et al., ASPLOS'14, PAPER.md
+ * §3.2).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load or call this.
+ * It shares no code, header, table or helper with the CUDA library under
+ * paper_conf_asplos_samadijlm14_b200/ and include/; neither includes or links
+ * the other.
+ *
+ * Arithmetic: inputs and weights are fp32; every sum is accumulated in fp64
+ * and outputs are fp64 (the paper never states a precision, S9).
+ * Loops follow the paper's definitions in order; no folding, blocking or
+ * reordering.  Frames are [n, h, w] row-major, contiguous.
+ *
+ * Parity status: every function below is pinned by tests/test_oracle_*.py
+ * (scipy library routines, hand tables, closed forms, brute force); none is
+ * "parity unpinned".  The index map for tiles larger than 5x5 follows reading
+ * S5 (lattice of anchors); parity with the paper there rests on that reading.
+ */
+#ifndef PARAPROX_ORACLE_H
+#define PARAPROX_ORACLE_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* schemes and metrics use the oracle's own numbering (same meaning as the
+ * library's, defined independently) */
+enum { OR_EXACT = 0, OR_ROW = 1, OR_COL = 2, OR_CENTER = 3 };
+enum { OR_MRE = 0, OR_L2 = 1, OR_PSNR = 2 };
+
+/* Reaching-distance rule for one axis of a tile of radius r (PAPER.md
+ * L1196-1218 §3.2.3): m[i + r] = offset whose value stands in for offset i,
+ * i in [-r, r].  Returns 0, or -1 on bad arguments. */
+int oracle_index_map(int r, int d, int* m);
+
+/* Scheme -> per-axis reaching distances (reading S3/S4 of DESIGN.md):
+ * exact (0,0), row (d,0), column (0,d), centre (d,d). */
+int oracle_scheme_reaches(int scheme, int reach, int* dy, int* dx);
+
+/* Exact stencil, the plain definition:
+ * E(y,x) = sum_i sum_j w[i][j] * X(clamp(y+i), clamp(x+j)). */
+int oracle_stencil_exact(const float* x, int n, int h, int w,
+                         const float* wgt, int ky, int kx, double* out);
+
+/* Approximate stencil by literal per-window substitution (L1144-1148,
+ * L1196-1218): build the tile W_p, replace each element by the element at
+ * its index-mapped offset, then apply the filter to the substituted tile. */
+int oracle_stencil_approx(const float* x, int n, int h, int w,
+                          const float* wgt, int ky, int kx,
+                          int dy, int dx, double* out);
+
+/* Separable filter w = wy (outer) wx: horizontal pass then vertical pass,
+ * each with the substituted (dy, dx) windows, fp64 intermediate. */
+int oracle_stencil_sep(const float* x, int n, int h, int w,
+                       const float* wy, int ky, const float* wx, int kx,
+                       int dy, int dx, double* out);
+
+/* Output quality of approx against exact over `count` elements (Table 1,
+ * L1644-1664; §4.2).  MRE / L2 -> 1 - error; PSNR -> dB. */
+int oracle_quality(const double* e, const double* a, long long count,
+                   int metric, double* quality);
+
+/* Tuner candidates in cost order (O7).  Writes up to `cap`
+ * (scheme, reach) pairs, returns the count (or -1). */
+int oracle_tune_candidates(int ky, int kx, int separable, int cap,
+                           int* schemes, int* reaches);
+
+/* TOQ tuner (L572-592 §2; L1220-1226 §3.2.4; L1620-1628 §4.1): run the exact
+ * kernel once and each candidate in cost order on the training frames; the
+ * first whose quality >= toq wins, else (EXACT, 0, 1.0).  Outputs are rounded
+ * to fp32 ("what the user gets") before the quality is taken.  Per-candidate
+ * qualities (in candidate order, up to the decision) go to `qualities` when
+ * non-NULL (capacity `cap`); `*n_evaluated` receives their count. */
+int oracle_tune(const float* x, int n, int h, int w, int separable,
+                const float* wgt_or_wy, int ky, const float* wx, int kx,
+                double toq, int metric, int cap, double* qualities,
+                int* n_evaluated, int* scheme, int* reach, double* quality);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

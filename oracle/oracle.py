@@ -1,0 +1,190 @@
+"""ctypes wrapper over ``liboracle.so`` (plain C, fp64; see ``oracle.h``).
+
+TEST INFRASTRUCTURE ONLY (see ``oracle/__init__.py``).  Every function cites
+the PAPER.md passage it follows in ``oracle.c``.  Inputs are fp32 numpy
+arrays (the seeded generators in ``workloads/``); outputs are fp64.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_HDR = os.path.join(_HERE, "oracle.h")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+EXACT, ROW, COL, CENTER = 0, 1, 2, 3
+MRE, L2, PSNR = 0, 1, 2
+SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "center": CENTER, "centre": CENTER}
+METRICS = {"mre": MRE, "l2": L2, "psnr": PSNR}
+SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center"}
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (-O2, OpenMP, no fast-math)."""
+    stale = not os.path.exists(_LIB) or max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)) > os.path.getmtime(_LIB)
+    if force or stale:
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+                               "-Wall", "-Wextra", "-Wno-unused-parameter",
+                               _SRC, "-o", tmp, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(build())
+        P = C.POINTER
+        f32, f64, i32 = P(C.c_float), P(C.c_double), P(C.c_int)
+        _lib.oracle_index_map.argtypes = [C.c_int, C.c_int, i32]
+        _lib.oracle_scheme_reaches.argtypes = [C.c_int, C.c_int, i32, i32]
+        _lib.oracle_stencil_exact.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, C.c_int, f64]
+        _lib.oracle_stencil_approx.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, C.c_int,
+                                               C.c_int, C.c_int, f64]
+        _lib.oracle_stencil_sep.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                            C.c_int, C.c_int, f64]
+        _lib.oracle_quality.argtypes = [f64, f64, C.c_longlong, C.c_int, f64]
+        _lib.oracle_tune_candidates.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, i32, i32]
+        _lib.oracle_tune.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                     C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
+        for name in ("oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
+                     "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
+                     "oracle_tune_candidates", "oracle_tune"):
+            getattr(_lib, name).restype = C.c_int
+    return _lib
+
+
+def _fp(a):
+    return a.ctypes.data_as(C.POINTER(C.c_float))
+
+
+def _dp(a):
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _frames(x):
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    if x.ndim == 2:
+        return x[None], True
+    if x.ndim != 3:
+        raise ValueError("expected [h, w] or [n, h, w]")
+    return x, False
+
+
+def _ok(rc, what):
+    if rc != 0:
+        raise ValueError(f"oracle: {what} rejected its arguments")
+
+
+def index_map(r: int, d: int) -> np.ndarray:
+    """m[i + r] for i in [-r, r] (§3.2.3; reading S5)."""
+    m = np.zeros(2 * r + 1, dtype=np.int32)
+    _ok(lib().oracle_index_map(r, d, m.ctypes.data_as(C.POINTER(C.c_int))), "index_map")
+    return m
+
+
+def scheme_reaches(scheme, reach: int):
+    s = SCHEMES[scheme] if isinstance(scheme, str) else int(scheme)
+    dy, dx = C.c_int(), C.c_int()
+    _ok(lib().oracle_scheme_reaches(s, reach, C.byref(dy), C.byref(dx)), "scheme_reaches")
+    return dy.value, dx.value
+
+
+def stencil_exact(x, w) -> np.ndarray:
+    """E = sum_ij w[i][j] X(clamp(y+i), clamp(x+j)) in fp64."""
+    x, squeeze = _frames(x)
+    w = np.ascontiguousarray(w, dtype=np.float32)
+    out = np.empty(x.shape, dtype=np.float64)
+    n, h, ww = x.shape
+    _ok(lib().oracle_stencil_exact(_fp(x), n, h, ww, _fp(w), w.shape[0], w.shape[1], _dp(out)),
+        "stencil_exact")
+    return out[0] if squeeze else out
+
+
+def stencil_approx_xy(x, w, dy: int, dx: int) -> np.ndarray:
+    """Literal per-window substitution with per-axis reaches (dy, dx)."""
+    x, squeeze = _frames(x)
+    w = np.ascontiguousarray(w, dtype=np.float32)
+    out = np.empty(x.shape, dtype=np.float64)
+    n, h, ww = x.shape
+    _ok(lib().oracle_stencil_approx(_fp(x), n, h, ww, _fp(w), w.shape[0], w.shape[1], dy, dx, _dp(out)),
+        "stencil_approx")
+    return out[0] if squeeze else out
+
+
+def stencil_approx(x, w, scheme, reach: int) -> np.ndarray:
+    dy, dx = scheme_reaches(scheme, reach)
+    return stencil_approx_xy(x, w, dy, dx)
+
+
+def stencil_sep(x, wy, wx, dy: int = 0, dx: int = 0) -> np.ndarray:
+    x, squeeze = _frames(x)
+    wy = np.ascontiguousarray(wy, dtype=np.float32).ravel()
+    wx = np.ascontiguousarray(wx, dtype=np.float32).ravel()
+    out = np.empty(x.shape, dtype=np.float64)
+    n, h, ww = x.shape
+    _ok(lib().oracle_stencil_sep(_fp(x), n, h, ww, _fp(wy), wy.size, _fp(wx), wx.size, dy, dx, _dp(out)),
+        "stencil_sep")
+    return out[0] if squeeze else out
+
+
+def stencil_sep_scheme(x, wy, wx, scheme, reach: int) -> np.ndarray:
+    dy, dx = scheme_reaches(scheme, reach)
+    return stencil_sep(x, wy, wx, dy, dx)
+
+
+def quality(e, a, metric="mre") -> float:
+    """1 - MRE / 1 - L2 (Table 1) or PSNR dB (not a paper metric)."""
+    m = METRICS[metric] if isinstance(metric, str) else int(metric)
+    e = np.ascontiguousarray(e, dtype=np.float64).ravel()
+    a = np.ascontiguousarray(a, dtype=np.float64).ravel()
+    if e.size != a.size:
+        raise ValueError("size mismatch")
+    q = C.c_double()
+    _ok(lib().oracle_quality(_dp(e), _dp(a), e.size, m, C.byref(q)), "quality")
+    return q.value
+
+
+def tune_candidates(ky: int, kx: int, separable: bool = False):
+    cap = 64
+    s = np.zeros(cap, dtype=np.int32)
+    r = np.zeros(cap, dtype=np.int32)
+    n = lib().oracle_tune_candidates(ky, kx, int(separable), cap,
+                                     s.ctypes.data_as(C.POINTER(C.c_int)),
+                                     r.ctypes.data_as(C.POINTER(C.c_int)))
+    if n < 0:
+        raise ValueError("tune_candidates rejected its arguments")
+    return [(SCHEME_NAMES[int(s[i])], int(r[i])) for i in range(n)]
+
+
+def tune(x, w, toq: float, metric="mre", all_qualities: bool = False):
+    """Oracle tuner.  ``w`` is a 2-D array (dense) or a (wy, wx) pair
+    (separable).  Returns dict(scheme, reach, quality, qualities)."""
+    x, _ = _frames(x)
+    m = METRICS[metric] if isinstance(metric, str) else int(metric)
+    n, h, ww = x.shape
+    if isinstance(w, (tuple, list)):
+        wy = np.ascontiguousarray(w[0], dtype=np.float32).ravel()
+        wx = np.ascontiguousarray(w[1], dtype=np.float32).ravel()
+        sep, ky, kx, wa, wb = 1, wy.size, wx.size, wy, wx
+    else:
+        wa = np.ascontiguousarray(w, dtype=np.float32)
+        sep, ky, kx, wb = 0, wa.shape[0], wa.shape[1], wa
+    cap = 64
+    qs = np.full(cap, np.nan)
+    nev, sc, rc = C.c_int(), C.c_int(), C.c_int()
+    q = C.c_double()
+    _ok(lib().oracle_tune(_fp(x), n, h, ww, sep, _fp(wa), ky, _fp(wb), kx, float(toq), m, cap,
+                          _dp(qs) if all_qualities else None, C.byref(nev), C.byref(sc), C.byref(rc),
+                          C.byref(q)), "tune")
+    return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value,
+                qualities=[float(v) for v in qs[:nev.value]] if all_qualities else None)
