@@ -1,0 +1,429 @@
+#!/usr/bin/env python
+"""Benchmark of the Paraprox Stencil & Partition hot path on B200.
+
+Metric (BASELINE.json): Mpixel/s and HBM GB/s of the approximate stencil vs
+the exact stencil at TOQ = 90%, on 1/2/4/8 B200.
+
+A step is one pass of the deployed hot path over one batch: the approximate
+stencil at the (scheme, reach) the TOQ tuner chose.  The plan (a1) and the
+tuner (a5) run once before the timed region on the 10 training frames, as in
+the paper ("We ran the first 10 executions to train and detect the best
+kernel, and then we measured ... the next 100 executions", PAPER.md
+L1620-1628); the exact stencil (a2) is timed the same way in the same run for
+the speedup, and the quality (a4) of the chosen configuration is measured on
+the held-out frames.  DESIGN.md "Measurement" has the details.
+
+Default workload c2 (BASELINE.json configs[1]): 4096x4096 fp32, 5x5 mean, MRE.
+Weak scaling: every rank processes its own frames; no collective on the data
+path (a barrier brackets the timed region; times are max over ranks).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Mpixel/s and HBM GB/s (approx vs exact) at TOQ=90%, 1/2/4/8 B200"
+
+WORKLOADS = {
+    # name: frames per step, h, w, filter, metric, description
+    "c2": dict(n=1, h=4096, w=4096, filter="mean5", metric="mre",
+               desc="4096x4096 fp32, 5x5 mean filter (BASELINE configs[1])"),
+    "c1": dict(n=110, h=512, w=512, filter="gauss3", metric="mre",
+               desc="110 frames 512x512 fp32, 3x3 Gaussian (configs[0], batched)"),
+    "c3": dict(n=256, h=2160, w=3840, filter="sep7", metric="l2",
+               desc="256 frames 3840x2160 fp32, 7x7 separable (configs[2])"),
+    "c4": dict(n=1, h=32768, w=32768, filter="conv9", metric="l2",
+               desc="32768x32768 fp32, 9x9 convolution (configs[3])"),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def load_traffic(workload, kernel):
+    """dram bytes per launch from a committed ncu --set full capture, if any."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        d = json.load(open(p))
+        return d.get(workload, {}).get(kernel)
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons while the GPU is busy."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, index, period=0.002):
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._period = period
+        self._ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self._ok = True
+        except Exception as e:  # pragma: no cover
+            self.error = str(e)
+
+    def _run(self):
+        nv = self._nv
+        while not self._stop.is_set():
+            try:
+                mhz = nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM)
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                self.samples.append(mhz)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self._period)
+
+    def __enter__(self):
+        if self._ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self._ok:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self._ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": len(self.samples)}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def make_filter_arrays(name):
+    from workloads import filters as F
+    kind, w = F.named(name)
+    return kind, w
+
+
+def oracle_run(x, kind, w, scheme, reach):
+    import oracle
+    if kind == "sep":
+        return oracle.stencil_sep_scheme(x, w[0], w[1], scheme, reach)
+    return oracle.stencil_approx(x, w, scheme, reach)
+
+
+def cpu_baseline(wl, kind, w, scheme, reach, budget_s=12.0, max_reps=16):
+    """The oracle as it stands, on the host cores, over a bounded sample of the
+    workload: whole frames (or a row band of the c4 image) until ~budget_s."""
+    import oracle
+    import workloads as W
+    cores = int(os.environ.get("OMP_NUM_THREADS", len(os.sched_getaffinity(0))))
+    h, wd = wl["h"], wl["w"]
+    rows = h if h * wd <= 4096 * 4096 else 1024
+    x = W.image(rows, wd, 1000) if rows == h else W.periodic(rows, wd, tile=4096, seed=0)
+    oracle.lib()
+    px = 0
+    t0 = time.perf_counter()
+    reps = 0
+    while reps < max_reps:
+        oracle_run(x, kind, w, scheme, reach)
+        px += x.size
+        reps += 1
+        if time.perf_counter() - t0 >= budget_s:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": px / dt / 1e6, "unit": "Mpixel/s", "cores": cores, "kind": "oracle",
+            "sample": f"{reps} x {rows}x{wd} frame(s), {scheme}:{reach}, fp64 literal per-window oracle",
+            "seconds": dt}
+
+
+def dist_setup():
+    import torch
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        return dist, rank, ws, local
+    return None, 0, 1, local
+
+
+def run_reference(args):
+    """--impl reference: the oracle (the slow plain CPU program) on this box's
+    host cores, rank 0 only, each step a bounded sample of the workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import workloads as W
+    import oracle
+    wl = WORKLOADS[args.workload]
+    kind, w = make_filter_arrays(wl["filter"])
+    cores = int(os.environ.get("OMP_NUM_THREADS", len(os.sched_getaffinity(0))))
+    # bounded sample per step: a 512-row band of the frame, at the scheme the
+    # oracle tuner picks at the TOQ on a small training set (2 frames, 512 rows)
+    band = min(wl["h"], 512)
+    x = W.image(band, wl["w"], 2000) if wl["h"] * wl["w"] <= 4096 * 4096 else \
+        W.periodic(band, wl["w"], tile=4096, seed=0)
+    train = W.frames(2, 512, min(wl["w"], 4096), 0)
+    res = oracle.tune(train, w, args.toq, wl["metric"])
+    scheme, reach = res["scheme"], res["reach"]
+    for _ in range(args.warmup):
+        oracle_run(x[:64], kind, w, scheme, reach)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle_run(x, kind, w, scheme, reach)
+        times.append(time.perf_counter() - t0)
+    dt = sum(times)
+    value = x.size * args.steps / dt / 1e6
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "Mpixel/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.workload, "desc": wl["desc"], "sample_rows": band, "scheme": scheme,
+                   "reach": reach, "toq": args.toq},
+        "cpu_baseline": {"value": value, "unit": "Mpixel/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{band}x{wl['w']} band per step of {args.workload}"},
+        "e2e": {"value": value, "unit": "Mpixel/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS))
+    ap.add_argument("--toq", type=float, default=0.90)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import paper_conf_asplos_samadijlm14_b200 as pkg
+    import workloads as W
+    P = pkg.paraprox
+
+    dist, rank, ws, local = dist_setup()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    wl = WORKLOADS[args.workload]
+    kind, w = make_filter_arrays(wl["filter"])
+    f = P.Filter(wy=w[0], wx=w[1]) if kind == "sep" else P.Filter(w)
+    n, h, wd = wl["n"], wl["h"], wl["w"]
+    px_step = n * h * wd
+
+    # ---- inputs: training frames (tuner), held-out frames (timed) ----------
+    seed_base = 1000 * rank
+    tn = 10 if h * wd <= 4096 * 4096 else 2
+    th, tw = (h, wd) if h * wd <= 4096 * 4096 else (4096, 4096)
+    train = torch.from_numpy(W.frames(tn, th, tw, seed_base)).to(dev)
+    if args.workload == "c4":
+        held = [torch.from_numpy(W.periodic(h, wd, tile=4096, seed=seed_base + 10)).to(dev).view(1, h, wd)]
+    elif n == 1:
+        distinct = [torch.from_numpy(W.image(h, wd, seed_base + 10 + k)).to(dev).view(1, h, wd) for k in range(2)]
+        held = distinct
+    else:
+        distinct = W.frames(min(n, 16), h, wd, seed_base + 10)
+        t = torch.empty((n, h, wd), device=dev)
+        for k in range(n):
+            t[k].copy_(torch.from_numpy(distinct[k % len(distinct)]))
+        held = [t]
+    # rotate over enough buffers that consecutive steps never hit in L2
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    nbuf = max(1, min(8, -(-(3 * l2) // (8 * px_step))))
+    inputs = [held[k % len(held)] if k < len(held) else held[k % len(held)].clone() for k in range(nbuf)]
+    outputs = [torch.empty_like(inputs[0]) for _ in range(nbuf)]
+
+    # ---- tune once (paper: first 10 executions train) ----------------------
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    if ws > 1:
+        parts = P.tune_partials(train, f, wl["metric"])
+        pt = torch.from_numpy(parts).to(dev)
+        dist.all_reduce(pt)
+        scheme, reach, q_train = P.tune_decide(f, pt.cpu().numpy(), args.toq, wl["metric"])
+    else:
+        scheme, reach, q_train = P.tune(train, f, args.toq, wl["metric"])
+    tune_ms = 1e3 * (time.perf_counter() - t0)
+    del train
+    plan = f.plan_info(*{"exact": (0, 0), "row": (reach, 0), "col": (0, reach),
+                         "center": (reach, reach)}[scheme])
+
+    def timed(fn, steps, warmup):
+        for k in range(warmup):
+            fn(k)
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        t_all0 = torch.cuda.Event(enable_timing=True)
+        t_all1 = torch.cuda.Event(enable_timing=True)
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        l0 = P.launch_count()
+        t_all0.record(stream)
+        for k in range(steps):
+            starts[k].record(stream)
+            fn(k)
+            ends[k].record(stream)
+        t_all1.record(stream)
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        launches = P.launch_count() - l0
+        total = t_all0.elapsed_time(t_all1)
+        per = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+        tot = torch.tensor([total, sum(per)], device=dev, dtype=torch.float64)
+        if dist:
+            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        return float(tot[0]), float(tot[1]) / steps, launches
+
+    # arguments marshalled once per buffer: the loop is one ctypes call per step
+    approx_ops = [P.prepare(inputs[k], f, scheme, reach, outputs[k], stream=stream) for k in range(nbuf)]
+    exact_ops = [P.prepare(inputs[k], f, "exact", 0, outputs[k], stream=stream) for k in range(nbuf)]
+
+    def approx_step(k):
+        approx_ops[k % nbuf]()
+
+    def exact_step(k):
+        exact_ops[k % nbuf]()
+
+    with ClockSampler(local) as clk:
+        total_ms, kern_ms, launches = timed(approx_step, args.steps, args.warmup)
+        exact_total_ms, exact_kern_ms, _ = timed(exact_step, args.steps, args.warmup)
+    approx_kernel = P.last_kernel()
+
+    ms_step = total_ms / args.steps
+    value = px_step * ws / (ms_step * 1e-3) / 1e6
+    exact_ms_step = exact_total_ms / args.steps
+    exact_value = px_step * ws / (exact_ms_step * 1e-3) / 1e6
+    peak, peak_kind = load_peaks()
+    alg_bytes = 8.0 * px_step  # 4 B read + 4 B written per output pixel (DESIGN.md roofline)
+    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
+    exact_achieved = alg_bytes / (exact_kern_ms * 1e-3) / 1e9
+
+    # ---- quality of the chosen configuration on the held-out frames ---------
+    q_held = None
+    if scheme != "exact":
+        e = P.stencil_exact(inputs[0], f)
+        a = P.stencil_approx(inputs[0], f, scheme, reach)
+        q_held = P.quality(e, a, wl["metric"])
+        del e, a
+
+    # ---- end to end through the public API, host buffers --------------------
+    e2e = None
+    if args.e2e_steps > 0 and px_step * 4 <= (8 << 30):
+        hin = inputs[0].cpu().pin_memory()
+        hout = torch.empty_like(hin, pin_memory=True)
+        P.run_host(hin, f, scheme, reach, out=hout)  # warm
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        ev0 = torch.cuda.Event(enable_timing=True)
+        ev1 = torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for _ in range(args.e2e_steps):
+            P.run_host(hin, f, scheme, reach, out=hout)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+        t = torch.tensor([wall], device=dev, dtype=torch.float64)
+        if dist:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t[0]) / args.e2e_steps
+        e2e = {"value": px_step * ws / e2e_s / 1e6, "unit": "Mpixel/s", "h2d_bytes_per_step": 4 * px_step,
+               "d2h_bytes_per_step": 4 * px_step, "steps": args.e2e_steps,
+               "api": "paraprox_run_host (pinned host in/out; H2D, kernel, D2H overlapped in chunks)",
+               "timing": "host wall clock around synchronous calls, max over ranks"}
+        del hin, hout
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        try:
+            cpu = cpu_baseline(wl, kind, w, scheme, reach)
+        except Exception as ex:  # the oracle is a reported baseline, never the product path
+            cpu = {"value": None, "unit": "Mpixel/s", "cores": None, "kind": "oracle", "sample": f"failed: {ex}"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC,
+            "value": value,
+            "unit": "Mpixel/s",
+            "n_gpus": ws,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": ms_step,
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f32",
+            "data": "synthetic",
+            "config": {
+                "workload": args.workload, "desc": wl["desc"], "frames_per_step": n, "h": h, "w": wd,
+                "filter": wl["filter"], "toq": args.toq, "metric_quality": wl["metric"],
+                "l2_defeat": f"rotating {nbuf} input/output buffer pairs ({nbuf * 8 * px_step / 2**20:.0f} MiB "
+                             f"> 3x L2) so consecutive steps never hit in L2",
+                "parallelism": f"frames/replicas x{ws} (weak, no data-path collective)",
+            },
+            "hbm_gbs": alg_bytes * ws / (ms_step * 1e-3) / 1e9,
+            "tuned": {"scheme": scheme, "reach": reach, "quality_train": q_train, "quality_heldout": q_held,
+                      "taps": plan["taps"], "halo_y": plan["halo_y"], "halo_x": plan["halo_x"],
+                      "tune_ms": tune_ms, "train_frames": tn},
+            "exact": {"value": exact_value, "unit": "Mpixel/s", "ms_per_step": exact_ms_step,
+                      "hbm_gbs": alg_bytes * ws / (exact_ms_step * 1e-3) / 1e9,
+                      "kernel_gbs": exact_achieved, "roofline_frac": exact_achieved / peak},
+            "speedup_vs_exact": exact_ms_step / ms_step,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": load_traffic(args.workload, approx_kernel),
+                         "kernel": approx_kernel, "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
+                         "algorithmic_bytes_per_launch": alg_bytes, "avg_launch_ms": kern_ms},
+            "clocks": clk.summary(),
+            "gpu_launches": launches,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,201 @@
+/*
+ * paraprox.h -- C ABI of the B200-native Stencil & Partition approximation
+ * library (libparaprox.so).
+ *
+ * The method: Samadi, Jamshidi, Lee, Mahlke, "Paraprox: Pattern-Based
+ * Approximation for Data Parallel Applications", ASPLOS'14, §3.2 (PAPER.md
+ * L1118-1226).  A K_y x K_x stencil (Gaussian, mean, convolution filter) is
+ * approximated by reading only some elements of each output's tile: the
+ * centre, one row, or one column stands in for its neighbours up to a
+ * "reaching distance" (L1188-1218, Fig. 6), chosen by a runtime tuner so the
+ * output quality (Table 1 metrics, L1644-1664) meets a target output quality
+ * (TOQ, §4.2; runtime L572-592, training protocol L1620-1628).
+ *
+ * Conventions (all entry points):
+ *  - Images are fp32, row-major.  A paraprox_image describes n frames of
+ *    h x w elements; element (f, y, x) lives at base + f*frame_stride +
+ *    y*pitch + x (elements, not bytes).  Input and output buffers share the
+ *    descriptor.  Borders are clamped to the edge (reading S7).
+ *  - halo_top / halo_bottom (input only): that many valid rows exist above
+ *    row 0 / below row h-1 of every input frame (row-stripe decomposition);
+ *    clamping happens at the edge of the valid rows, so an interior stripe
+ *    with halos >= the filter radius computes exactly the rows the whole image
+ *    would.  0 = clamp at that edge.  Outputs cover rows 0..h-1 only.
+ *  - Device pointers ("d_") are caller-owned CUDA device memory; host
+ *    pointers ("h_") are caller-owned host memory.  The library owns filter
+ *    handles and nothing else; scratch comes from cudaMallocAsync on the
+ *    caller's stream and is released before return (stream-ordered).
+ *  - Streams: paraprox_stream is a cudaStream_t (NULL = legacy default
+ *    stream).  Stencil calls are asynchronous with respect to the host;
+ *    calls documented "syncs s" return after the stream has drained.
+ *  - d_out must not overlap the input rows that are read (no in-place).
+ *  - Errors are returned as paraprox_status codes; nothing aborts or throws.
+ *    paraprox_last_error() gives a thread-local detail string.  Execution
+ *    errors of asynchronous kernels surface at the caller's next sync.
+ *  - There is no CPU fallback: every computation runs in this library's
+ *    sm_100a kernels.
+ */
+#ifndef PARAPROX_H
+#define PARAPROX_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PARAPROX_VERSION 1
+#define PARAPROX_MAX_K 17 /* largest tile: the paper's 1x17 ConvSep loops (L1920-1922) */
+
+#if defined(__GNUC__)
+#define PARAPROX_API __attribute__((visibility("default")))
+#else
+#define PARAPROX_API
+#endif
+
+typedef struct CUstream_st* paraprox_stream;       /* == cudaStream_t */
+typedef struct paraprox_filter_s* paraprox_filter; /* opaque, library-owned, immutable */
+
+typedef enum {
+    PARAPROX_OK = 0,
+    PARAPROX_ERR_INVALID_ARG = 1, /* null pointer, even/non-positive K, reach < 0,
+                                     n/h/w < 1, pitch < w, overlap, bad TOQ, bad enum */
+    PARAPROX_ERR_UNSUPPORTED = 2, /* K > PARAPROX_MAX_K */
+    PARAPROX_ERR_CUDA = 3,        /* a CUDA runtime call or kernel launch failed */
+    PARAPROX_ERR_ALLOC = 4        /* host or device allocation failed */
+} paraprox_status;
+
+/* Fig. 6 (L1156-1166): exact; row (rows within the reach copy the accessed
+ * row); column; centre (the tile centre stands in for its neighbours). */
+typedef enum {
+    PARAPROX_EXACT = 0,
+    PARAPROX_ROW = 1,
+    PARAPROX_COL = 2,
+    PARAPROX_CENTER = 3
+} paraprox_scheme;
+
+/* Table 1 (L1644-1664): mean relative error (Gaussian, mean filters) and
+ * L2-norm (Convolution Separable); quality = 1 - error.  PSNR (dB) is offered
+ * as a reported metric and is not a paper metric (reading S11). */
+typedef enum { PARAPROX_MRE = 0, PARAPROX_L2 = 1, PARAPROX_PSNR = 2 } paraprox_metric;
+
+typedef struct {
+    int n, h, w;             /* frames, rows, columns (>= 1)                 */
+    long long pitch;         /* elements between rows (>= w)                 */
+    long long frame_stride;  /* elements between frames
+                                (>= (h + halo_top + halo_bottom) * pitch)     */
+    int halo_top, halo_bottom; /* valid input rows above / below (>= 0)      */
+} paraprox_image;
+
+/* ---- filters ---------------------------------------------------------- */
+
+/* Dense K_y x K_x weights, row-major, applied as a correlation (S8):
+ * out(y,x) = sum_{i,j} w[i][j] * in(y + i - K_y/2, x + j - K_x/2).
+ * K_y, K_x odd, 1..PARAPROX_MAX_K.  The weights are copied. */
+PARAPROX_API paraprox_status paraprox_filter_create(int ky, int kx, const float* h_w, paraprox_filter* out);
+
+/* Separable weights w = w_y (outer) w_x, computed as a fused horizontal then
+ * vertical pass (ConvSep, Table 1).  The weights are copied. */
+PARAPROX_API paraprox_status paraprox_filter_create_separable(int ky, const float* h_wy, int kx,
+                                                 const float* h_wx, paraprox_filter* out);
+
+PARAPROX_API void paraprox_filter_destroy(paraprox_filter f);
+
+PARAPROX_API paraprox_status paraprox_filter_shape(paraprox_filter f, int* ky, int* kx, int* separable);
+
+/* Plan introspection for per-axis reaches (reach_y, reach_x): the number of
+ * taps the kernel evaluates (|Ry|*|Rx| dense, |Ry|+|Rx| separable), the
+ * vertical/horizontal halo (largest accessed offset), and the per-axis index
+ * maps m_y[0..K_y-1], m_x[0..K_x-1] (offset of the element read in place of
+ * offset i - K/2; may be NULL).  Host-only. */
+PARAPROX_API paraprox_status paraprox_plan_info(paraprox_filter f, int reach_y, int reach_x, int* taps,
+                                   int* halo_y, int* halo_x, int* h_map_y, int* h_map_x);
+
+/* ---- stencils (asynchronous on s) ------------------------------------- */
+
+/* Exact stencil, every tap of every tile (the baseline, L544-552). */
+PARAPROX_API paraprox_status paraprox_stencil_exact(paraprox_filter f, const float* d_in, float* d_out,
+                                       const paraprox_image* img, paraprox_stream s);
+
+/* Approximate stencil with a scheme and a reaching distance (L1188-1218).
+ * reach > K/2 saturates; reach 0 or PARAPROX_EXACT computes the exact stencil.
+ * Separable filters: row -> vertical pass approximated, column -> horizontal,
+ * centre -> both ("reaching distances of both loops", L2110-2112). */
+PARAPROX_API paraprox_status paraprox_stencil_approx(paraprox_filter f, paraprox_scheme scheme, int reach,
+                                        const float* d_in, float* d_out,
+                                        const paraprox_image* img, paraprox_stream s);
+
+/* Per-axis reaching distances: row = (d, 0), column = (0, d), centre = (d, d). */
+PARAPROX_API paraprox_status paraprox_stencil_approx_xy(paraprox_filter f, int reach_y, int reach_x,
+                                           const float* d_in, float* d_out,
+                                           const paraprox_image* img, paraprox_stream s);
+
+/* End-to-end convenience over HOST buffers: copies h_in to the device,
+ * runs the stencil (scheme, reach), copies the result to h_out, overlapping
+ * the transfers with the kernels chunk by chunk.  Pinned host memory gives
+ * asynchronous copies; pageable memory works but serialises.  halo_top and
+ * halo_bottom must be 0.  Syncs s. */
+PARAPROX_API paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int reach,
+                                  const float* h_in, float* h_out, const paraprox_image* img,
+                                  paraprox_stream s);
+
+/* ---- output quality (syncs s) ------------------------------------------ */
+
+/* Quality of d_approx against d_exact over all n*h*w elements (pooled over
+ * frames, S12): 1 - MRE, 1 - L2 or PSNR dB.  fp64 accumulation in a fixed
+ * order: the result is deterministic for a given image shape. */
+PARAPROX_API paraprox_status paraprox_quality(const float* d_exact, const float* d_approx,
+                                 const paraprox_image* img, paraprox_metric m,
+                                 double* h_quality, paraprox_stream s);
+
+/* The 3 fp64 partial sums behind paraprox_quality (MRE: sum of relative
+ * errors, count, 0; L2: sum (A-E)^2, sum E^2, count; PSNR: sum (A-E)^2,
+ * count, 0).  Partials of disjoint pixel sets add (multi-GPU all-reduce). */
+PARAPROX_API paraprox_status paraprox_quality_partials(const float* d_exact, const float* d_approx,
+                                          const paraprox_image* img, paraprox_metric m,
+                                          double* h_partials3, paraprox_stream s);
+
+/* Quality from (summed) partials.  Host-only. */
+PARAPROX_API paraprox_status paraprox_quality_from_partials(const double* h_partials3, paraprox_metric m,
+                                               double* h_quality);
+
+/* ---- TOQ tuner (syncs s) ------------------------------------------------ */
+
+/* The runtime tuner (L572-592; L1220-1226; training on the first frames,
+ * L1620-1628): the exact kernel runs once on the training frames d_train,
+ * every candidate (scheme, reach) in cost order runs and is scored; the
+ * first candidate with quality >= toq is returned, else (EXACT, 0, 1.0 or
+ * +inf dB).  toq in (0, 1] for MRE / L2; any value (dB) for PSNR. */
+PARAPROX_API paraprox_status paraprox_tune(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                              double toq, paraprox_metric m, paraprox_scheme* out_scheme,
+                              int* out_reach, double* out_quality, paraprox_stream s);
+
+/* Candidates in cost order (O7).  *n receives the count; at most
+ * cap entries are written (schemes/reaches may be NULL to query the count). */
+PARAPROX_API paraprox_status paraprox_tune_candidates(paraprox_filter f, int cap, int* n,
+                                         paraprox_scheme* schemes, int* reaches);
+
+/* Multi-GPU split of paraprox_tune: 3 quality partials per candidate (in
+ * candidate order, 3*n doubles) for the local training frames ... */
+PARAPROX_API paraprox_status paraprox_tune_partials(paraprox_filter f, const float* d_train,
+                                       const paraprox_image* img, paraprox_metric m,
+                                       double* h_partials, paraprox_stream s);
+
+/* ... and the host-only decision from (all-reduced) partials.  Every rank
+ * holding the same summed partials reaches the same decision. */
+PARAPROX_API paraprox_status paraprox_tune_decide(paraprox_filter f, const double* h_partials,
+                                     paraprox_metric m, double toq, paraprox_scheme* out_scheme,
+                                     int* out_reach, double* out_quality);
+
+/* ---- diagnostics -------------------------------------------------------- */
+
+PARAPROX_API const char* paraprox_status_string(paraprox_status st);
+PARAPROX_API const char* paraprox_last_error(void);       /* thread-local detail of the last failure */
+PARAPROX_API int paraprox_version(void);
+/* Kernels this library has launched since load (all threads). */
+PARAPROX_API unsigned long long paraprox_launch_count(void);
+/* Name of the kernel variant the last stencil call on this thread used. */
+PARAPROX_API const char* paraprox_last_kernel(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PARAPROX_H */

@@ -1,0 +1,468 @@
+// api.cpp -- the extern "C" entry points of libparaprox (include/paraprox.h):
+// argument validation, plan lookup, stream-ordered scratch, the TOQ tuner and
+// the host-buffer end-to-end path.  All arithmetic runs in the kernels.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "internal.h"
+
+namespace ppx {
+
+std::atomic<unsigned long long> g_launches{0};
+thread_local const char* t_last_kernel = "none";
+static thread_local std::string t_err;
+
+void count_launch(const char* name) {
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    t_last_kernel = name;
+}
+
+static paraprox_status fail(paraprox_status st, const std::string& msg) {
+    t_err = msg;
+    return st;
+}
+
+static paraprox_status cuda_fail(cudaError_t e, const char* where) {
+    t_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return e == cudaErrorMemoryAllocation ? PARAPROX_ERR_ALLOC : PARAPROX_ERR_CUDA;
+}
+
+#define PPX_CUDA(call)                                  \
+    do {                                                \
+        cudaError_t _e = (call);                        \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call); \
+    } while (0)
+
+static bool odd_k(int k) { return k >= 1 && (k & 1) == 1; }
+
+static paraprox_status check_image(const paraprox_image* img, bool allow_halo) {
+    if (!img) return fail(PARAPROX_ERR_INVALID_ARG, "img is NULL");
+    if (img->n < 1 || img->h < 1 || img->w < 1) return fail(PARAPROX_ERR_INVALID_ARG, "n, h, w must be >= 1");
+    if (img->pitch < img->w) return fail(PARAPROX_ERR_INVALID_ARG, "pitch < w");
+    if (img->halo_top < 0 || img->halo_bottom < 0) return fail(PARAPROX_ERR_INVALID_ARG, "negative halo");
+    if (!allow_halo && (img->halo_top || img->halo_bottom))
+        return fail(PARAPROX_ERR_INVALID_ARG, "halos not allowed here");
+    const long long rows = (long long)img->h + img->halo_top + img->halo_bottom;
+    if (img->n > 1 && img->frame_stride < rows * img->pitch)
+        return fail(PARAPROX_ERR_INVALID_ARG, "frame_stride < (h + halos) * pitch");
+    return PARAPROX_OK;
+}
+
+static View view_of(const paraprox_image* img) {
+    View v;
+    v.n = img->n;
+    v.h = img->h;
+    v.w = img->w;
+    v.pitch = img->pitch;
+    v.fstride = img->n > 1 ? img->frame_stride : (long long)(img->h + img->halo_bottom) * img->pitch;
+    v.lo = -img->halo_top;
+    v.hi = img->h - 1 + img->halo_bottom;
+    return v;
+}
+
+// byte ranges touched: inputs (with halos) and outputs must not overlap
+static bool overlaps(const float* in, const float* out, const paraprox_image* img) {
+    const long long fs = img->n > 1 ? img->frame_stride : 0;
+    const char* i0 = (const char*)(in - (long long)img->halo_top * img->pitch);
+    const char* i1 = (const char*)(in + (img->n - 1) * fs + (long long)(img->h - 1 + img->halo_bottom) * img->pitch + img->w);
+    const char* o0 = (const char*)out;
+    const char* o1 = (const char*)(out + (img->n - 1) * fs + (long long)(img->h - 1) * img->pitch + img->w);
+    return i0 < o1 && o0 < i1;
+}
+
+static paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
+                                   const paraprox_image* img, paraprox_stream s) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    if (!in || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL buffer");
+    if (dy < 0 || dx < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    paraprox_status st = check_image(img, true);
+    if (st != PARAPROX_OK) return st;
+    if (overlaps(in, out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_in");
+    const Plan& p = get_plan(f, dy, dx);
+    const View v = view_of(img);
+    const long long ofs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
+    cudaError_t e = launch_stencil(p, in, v, out, img->pitch, ofs, (cudaStream_t)s);
+    if (e != cudaSuccess) return cuda_fail(e, "stencil launch");
+    return PARAPROX_OK;
+}
+
+static double quality_of(const double* p3, paraprox_metric m) {
+    if (m == PARAPROX_MRE) return 1.0 - p3[0] / p3[1];
+    if (m == PARAPROX_L2) {
+        if (p3[1] == 0.0) return p3[0] == 0.0 ? 1.0 : -INFINITY;
+        return 1.0 - std::sqrt(p3[0] / p3[1]);
+    }
+    const double mse = p3[0] / p3[1];
+    return mse == 0.0 ? INFINITY : 10.0 * std::log10(255.0 * 255.0 / mse);
+}
+
+static bool metric_ok(paraprox_metric m) { return m == PARAPROX_MRE || m == PARAPROX_L2 || m == PARAPROX_PSNR; }
+
+// scratch for one quality reduction: 2*kQualityBlocks partials + 3 results
+struct DevBuf {
+    void* p = nullptr;
+    cudaStream_t s = nullptr;
+    ~DevBuf() {
+        if (p) cudaFreeAsync(p, s);
+    }
+};
+
+static paraprox_status quality_partials_impl(const float* e, const float* a, const paraprox_image* img,
+                                             paraprox_metric m, double* h3, paraprox_stream s) {
+    if (!e || !a || !h3) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    cudaStream_t cs = (cudaStream_t)s;
+    DevBuf buf;
+    buf.s = cs;
+    PPX_CUDA(cudaMallocAsync(&buf.p, sizeof(double) * (2 * kQualityBlocks + 3), cs));
+    double* d = (double*)buf.p;
+    cudaError_t err = launch_quality(e, a, view_of(img), m, d + 2 * kQualityBlocks, d, cs);
+    if (err != cudaSuccess) return cuda_fail(err, "quality launch");
+    PPX_CUDA(cudaMemcpyAsync(h3, d + 2 * kQualityBlocks, 3 * sizeof(double), cudaMemcpyDeviceToHost, cs));
+    PPX_CUDA(cudaStreamSynchronize(cs));
+    return PARAPROX_OK;
+}
+
+// all candidates' partials into h_partials[3 * n]
+static paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                                          paraprox_metric m, const std::vector<Candidate>& cands,
+                                          double* h_partials, paraprox_stream s) {
+    if (!f || !d_train || (!h_partials && !cands.empty())) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    paraprox_status st = check_image(img, true);
+    if (st != PARAPROX_OK) return st;
+    if (cands.empty()) return PARAPROX_OK;
+    cudaStream_t cs = (cudaStream_t)s;
+    const long long plane = (long long)img->h * img->w;
+    const long long count = plane * img->n;
+    const size_t nc = cands.size();
+    DevBuf buf;
+    buf.s = cs;
+    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (2 * kQualityBlocks + 3 * nc) + 256;
+    PPX_CUDA(cudaMallocAsync(&buf.p, bytes, cs));
+    float* E = (float*)buf.p;
+    float* A = E + count;
+    double* scratch = (double*)(((uintptr_t)(A + count) + 255) & ~(uintptr_t)255);
+    double* parts = scratch + 2 * kQualityBlocks;
+    const View vin = view_of(img);
+    View vq;  // compact layout of the scratch outputs
+    vq.n = img->n;
+    vq.h = img->h;
+    vq.w = img->w;
+    vq.pitch = img->w;
+    vq.fstride = plane;
+    vq.lo = 0;
+    vq.hi = img->h - 1;
+    cudaError_t e = launch_stencil(get_plan(f, 0, 0), d_train, vin, E, img->w, plane, cs);
+    if (e != cudaSuccess) return cuda_fail(e, "exact launch");
+    for (size_t k = 0; k < nc; ++k) {
+        e = launch_stencil(get_plan(f, cands[k].dy, cands[k].dx), d_train, vin, A, img->w, plane, cs);
+        if (e != cudaSuccess) return cuda_fail(e, "candidate launch");
+        e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);
+        if (e != cudaSuccess) return cuda_fail(e, "quality launch");
+    }
+    PPX_CUDA(cudaMemcpyAsync(h_partials, parts, sizeof(double) * 3 * nc, cudaMemcpyDeviceToHost, cs));
+    PPX_CUDA(cudaStreamSynchronize(cs));
+    return PARAPROX_OK;
+}
+
+static paraprox_status decide(const std::vector<Candidate>& cands, const double* parts, paraprox_metric m,
+                              double toq, paraprox_scheme* sc, int* reach, double* q) {
+    *sc = PARAPROX_EXACT;
+    *reach = 0;
+    *q = m == PARAPROX_PSNR ? INFINITY : 1.0;
+    for (size_t k = 0; k < cands.size(); ++k) {
+        const double qk = quality_of(parts + 3 * k, m);
+        if (qk >= toq) {
+            *sc = cands[k].scheme;
+            *reach = cands[k].reach;
+            *q = qk;
+            return PARAPROX_OK;
+        }
+    }
+    return PARAPROX_OK;
+}
+
+static paraprox_status check_toq(double toq, paraprox_metric m) {
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    if (m != PARAPROX_PSNR && !(toq > 0.0 && toq <= 1.0)) return fail(PARAPROX_ERR_INVALID_ARG, "toq not in (0, 1]");
+    if (std::isnan(toq)) return fail(PARAPROX_ERR_INVALID_ARG, "toq is NaN");
+    return PARAPROX_OK;
+}
+
+}  // namespace ppx
+
+using namespace ppx;
+
+extern "C" {
+
+paraprox_status paraprox_filter_create(int ky, int kx, const float* h_w, paraprox_filter* out) {
+    if (!h_w || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!odd_k(ky) || !odd_k(kx)) return fail(PARAPROX_ERR_INVALID_ARG, "K must be odd and >= 1");
+    if (ky > kMaxK || kx > kMaxK) return fail(PARAPROX_ERR_UNSUPPORTED, "K > 17");
+    paraprox_filter f = new (std::nothrow) paraprox_filter_s;
+    if (!f) return fail(PARAPROX_ERR_ALLOC, "filter allocation");
+    f->ky = ky;
+    f->kx = kx;
+    f->separable = false;
+    f->w.assign(h_w, h_w + (size_t)ky * kx);
+    *out = f;
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_filter_create_separable(int ky, const float* h_wy, int kx, const float* h_wx,
+                                                 paraprox_filter* out) {
+    if (!h_wy || !h_wx || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!odd_k(ky) || !odd_k(kx)) return fail(PARAPROX_ERR_INVALID_ARG, "K must be odd and >= 1");
+    if (ky > kMaxK || kx > kMaxK) return fail(PARAPROX_ERR_UNSUPPORTED, "K > 17");
+    paraprox_filter f = new (std::nothrow) paraprox_filter_s;
+    if (!f) return fail(PARAPROX_ERR_ALLOC, "filter allocation");
+    f->ky = ky;
+    f->kx = kx;
+    f->separable = true;
+    f->wy.assign(h_wy, h_wy + ky);
+    f->wx.assign(h_wx, h_wx + kx);
+    *out = f;
+    return PARAPROX_OK;
+}
+
+void paraprox_filter_destroy(paraprox_filter f) { delete f; }
+
+paraprox_status paraprox_filter_shape(paraprox_filter f, int* ky, int* kx, int* separable) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    if (ky) *ky = f->ky;
+    if (kx) *kx = f->kx;
+    if (separable) *separable = f->separable ? 1 : 0;
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_plan_info(paraprox_filter f, int reach_y, int reach_x, int* taps, int* halo_y,
+                                   int* halo_x, int* h_map_y, int* h_map_x) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    if (reach_y < 0 || reach_x < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    const Plan& p = get_plan(f, reach_y, reach_x);
+    if (taps) *taps = p.taps;
+    if (halo_y) *halo_y = p.hy;
+    if (halo_x) *halo_x = p.hx;
+    if (h_map_y) std::copy(p.my, p.my + p.ky, h_map_y);
+    if (h_map_x) std::copy(p.mx, p.mx + p.kx, h_map_x);
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_stencil_exact(paraprox_filter f, const float* d_in, float* d_out,
+                                       const paraprox_image* img, paraprox_stream s) {
+    return run_stencil(f, 0, 0, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_stencil_approx(paraprox_filter f, paraprox_scheme scheme, int reach, const float* d_in,
+                                        float* d_out, const paraprox_image* img, paraprox_stream s) {
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    return run_stencil(f, dy, dx, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_stencil_approx_xy(paraprox_filter f, int reach_y, int reach_x, const float* d_in,
+                                           float* d_out, const paraprox_image* img, paraprox_stream s) {
+    return run_stencil(f, reach_y, reach_x, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_quality(const float* d_exact, const float* d_approx, const paraprox_image* img,
+                                 paraprox_metric m, double* h_quality, paraprox_stream s) {
+    if (!h_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    double p3[3];
+    paraprox_status st = quality_partials_impl(d_exact, d_approx, img, m, p3, s);
+    if (st != PARAPROX_OK) return st;
+    *h_quality = quality_of(p3, m);
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_quality_partials(const float* d_exact, const float* d_approx, const paraprox_image* img,
+                                          paraprox_metric m, double* h_partials3, paraprox_stream s) {
+    return quality_partials_impl(d_exact, d_approx, img, m, h_partials3, s);
+}
+
+paraprox_status paraprox_quality_from_partials(const double* h_partials3, paraprox_metric m, double* h_quality) {
+    if (!h_partials3 || !h_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    *h_quality = quality_of(h_partials3, m);
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_tune_candidates(paraprox_filter f, int cap, int* n, paraprox_scheme* schemes,
+                                         int* reaches) {
+    if (!f || !n) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (cap < 0) return fail(PARAPROX_ERR_INVALID_ARG, "cap < 0");
+    std::vector<Candidate> c = candidates(f);
+    *n = (int)c.size();
+    for (int k = 0; k < (int)c.size() && k < cap; ++k) {
+        if (schemes) schemes[k] = c[k].scheme;
+        if (reaches) reaches[k] = c[k].reach;
+    }
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_tune_partials(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                                       paraprox_metric m, double* h_partials, paraprox_stream s) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    return tune_partials_impl(f, d_train, img, m, candidates(f), h_partials, s);
+}
+
+paraprox_status paraprox_tune_decide(paraprox_filter f, const double* h_partials, paraprox_metric m, double toq,
+                                     paraprox_scheme* out_scheme, int* out_reach, double* out_quality) {
+    if (!f || !out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    std::vector<Candidate> c = candidates(f);
+    if (!c.empty() && !h_partials) return fail(PARAPROX_ERR_INVALID_ARG, "NULL partials");
+    return decide(c, h_partials, m, toq, out_scheme, out_reach, out_quality);
+}
+
+paraprox_status paraprox_tune(paraprox_filter f, const float* d_train, const paraprox_image* img, double toq,
+                              paraprox_metric m, paraprox_scheme* out_scheme, int* out_reach,
+                              double* out_quality, paraprox_stream s) {
+    if (!f || !out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    std::vector<Candidate> c = candidates(f);
+    std::vector<double> parts(3 * c.size() + 3);
+    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s);
+    if (st != PARAPROX_OK) return st;
+    return decide(c, parts.data(), m, toq, out_scheme, out_reach, out_quality);
+}
+
+paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int reach, const float* h_in,
+                                  float* h_out, const paraprox_image* img, paraprox_stream s) {
+    if (!f || !h_in || !h_out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    if (overlaps(h_in, h_out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "h_out overlaps h_in");
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    const Plan& p = get_plan(f, dy, dx);
+    cudaStream_t cs = (cudaStream_t)s;
+    const int n = img->n, h = img->h, w = img->w;
+    const long long plane = (long long)h * w;
+    const long long hfs = n > 1 ? img->frame_stride : 0;
+    DevBuf buf;
+    buf.s = cs;
+    PPX_CUDA(cudaMallocAsync(&buf.p, sizeof(float) * 2 * plane * n, cs));
+    float* din = (float*)buf.p;
+    float* dout = din + plane * n;
+    // chunks: frames when batched, else row bands (halo rows come along)
+    const int chunks = n > 1 ? std::min(n, 8) : std::max(1, std::min(8, h / 512));
+    cudaStream_t up = nullptr, down = nullptr;
+    PPX_CUDA(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
+    cudaError_t err = cudaStreamCreateWithFlags(&down, cudaStreamNonBlocking);
+    if (err != cudaSuccess) {
+        cudaStreamDestroy(up);
+        return cuda_fail(err, "cudaStreamCreate");
+    }
+    std::vector<cudaEvent_t> ev(3 * chunks + 1, nullptr);
+    for (auto& e : ev)
+        if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    auto cleanup = [&]() {
+        cudaStreamSynchronize(down);
+        cudaStreamSynchronize(up);
+        for (auto& e : ev)
+            if (e) cudaEventDestroy(e);
+        cudaStreamDestroy(up);
+        cudaStreamDestroy(down);
+    };
+    auto bail = [&](cudaError_t e2, const char* where) {
+        cleanup();
+        return cuda_fail(e2, where);
+    };
+    if (err != cudaSuccess) return bail(err, "cudaEventCreate");
+    // the device scratch is stream-ordered on cs: make the copy streams wait for it
+    if ((err = cudaEventRecord(ev[3 * chunks], cs)) != cudaSuccess) return bail(err, "record");
+    if ((err = cudaStreamWaitEvent(up, ev[3 * chunks], 0)) != cudaSuccess) return bail(err, "wait");
+    const size_t rowb = sizeof(float) * w;
+    int copied = 0;  // rows of the single frame already uploaded
+    for (int c = 0; c < chunks; ++c) {
+        View v;
+        const float* kin;
+        float* kout;
+        if (n > 1) {
+            const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
+            for (int fr = f0; fr < f1; ++fr)
+                if ((err = cudaMemcpy2DAsync(din + fr * plane, rowb, h_in + fr * hfs, sizeof(float) * img->pitch,
+                                             rowb, h, cudaMemcpyHostToDevice, up)) != cudaSuccess)
+                    return bail(err, "H2D");
+            v = {f1 - f0, h, w, (long long)w, plane, 0, h - 1};
+            kin = din + f0 * plane;
+            kout = dout + f0 * plane;
+        } else {
+            const int r0 = (int)((long long)h * c / chunks), r1 = (int)((long long)h * (c + 1) / chunks);
+            const int need = std::min(h, r1 + p.hy);
+            if (need > copied) {
+                if ((err = cudaMemcpy2DAsync(din + (long long)copied * w, rowb, h_in + (long long)copied * img->pitch,
+                                             sizeof(float) * img->pitch, rowb, need - copied,
+                                             cudaMemcpyHostToDevice, up)) != cudaSuccess)
+                    return bail(err, "H2D");
+                copied = need;
+            }
+            v = {1, r1 - r0, w, (long long)w, (long long)(r1 - r0) * w, -r0, need - 1 - r0};
+            kin = din + (long long)r0 * w;
+            kout = dout + (long long)r0 * w;
+        }
+        if ((err = cudaEventRecord(ev[3 * c], up)) != cudaSuccess) return bail(err, "record");
+        if ((err = cudaStreamWaitEvent(cs, ev[3 * c], 0)) != cudaSuccess) return bail(err, "wait");
+        err = launch_stencil(p, kin, v, kout, w, v.n > 1 ? plane : (long long)v.h * w, cs);
+        if (err != cudaSuccess) return bail(err, "stencil launch");
+        if ((err = cudaEventRecord(ev[3 * c + 1], cs)) != cudaSuccess) return bail(err, "record");
+        if ((err = cudaStreamWaitEvent(down, ev[3 * c + 1], 0)) != cudaSuccess) return bail(err, "wait");
+        if (n > 1) {
+            const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
+            for (int fr = f0; fr < f1; ++fr)
+                if ((err = cudaMemcpy2DAsync(h_out + fr * hfs, sizeof(float) * img->pitch, dout + fr * plane, rowb,
+                                             rowb, h, cudaMemcpyDeviceToHost, down)) != cudaSuccess)
+                    return bail(err, "D2H");
+        } else {
+            const int r0 = (int)((long long)h * c / chunks), r1 = (int)((long long)h * (c + 1) / chunks);
+            if ((err = cudaMemcpy2DAsync(h_out + (long long)r0 * img->pitch, sizeof(float) * img->pitch,
+                                         dout + (long long)r0 * w, rowb, rowb, r1 - r0, cudaMemcpyDeviceToHost,
+                                         down)) != cudaSuccess)
+                return bail(err, "D2H");
+        }
+    }
+    // the scratch is freed on cs: order it after the last download
+    if ((err = cudaEventRecord(ev[3 * chunks - 1], down)) != cudaSuccess) return bail(err, "record");
+    if ((err = cudaStreamWaitEvent(cs, ev[3 * chunks - 1], 0)) != cudaSuccess) return bail(err, "wait");
+    err = cudaStreamSynchronize(down);
+    cleanup();
+    if (err != cudaSuccess) return cuda_fail(err, "D2H sync");
+    buf.p = nullptr;
+    PPX_CUDA(cudaFreeAsync(din, cs));
+    PPX_CUDA(cudaStreamSynchronize(cs));
+    return PARAPROX_OK;
+}
+
+const char* paraprox_status_string(paraprox_status st) {
+    switch (st) {
+    case PARAPROX_OK: return "ok";
+    case PARAPROX_ERR_INVALID_ARG: return "invalid argument";
+    case PARAPROX_ERR_UNSUPPORTED: return "unsupported";
+    case PARAPROX_ERR_CUDA: return "CUDA error";
+    case PARAPROX_ERR_ALLOC: return "allocation failed";
+    default: return "unknown status";
+    }
+}
+
+const char* paraprox_last_error(void) { return t_err.c_str(); }
+int paraprox_version(void) { return PARAPROX_VERSION; }
+unsigned long long paraprox_launch_count(void) { return g_launches.load(); }
+const char* paraprox_last_kernel(void) { return t_last_kernel; }
+
+}  // extern "C"

@@ -1,0 +1,87 @@
+// internal.h -- shared declarations of libparaprox (host plan + kernel launchers).
+// Not part of the ABI; see include/paraprox.h.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "../../include/paraprox.h"
+
+namespace ppx {
+
+constexpr int kMaxK = PARAPROX_MAX_K;
+constexpr int kMaxR = kMaxK / 2;            // 8
+constexpr int kMaxTaps = kMaxK * kMaxK;     // 289
+
+// One approximation plan: filter x per-axis reaching distances (dy, dx).
+// Built once on the host and cached in the filter.
+struct Plan {
+    int ky = 1, kx = 1, ry = 0, rx = 0;
+    bool separable = false;
+    int dy = 0, dx = 0;                 // reaches, saturated to the radius
+    int my[kMaxK] = {}, mx[kMaxK] = {}; // index maps, m[i + r]
+    int ny = 0, nx = 0;                 // |Ry|, |Rx| accessed offsets per axis
+    int ay[kMaxK] = {}, ax[kMaxK] = {}; // accessed offsets, ascending
+    int hy = 0, hx = 0;                 // halos = max |accessed offset|
+    uint32_t masky = 0, maskx = 0;      // bit (a + kMaxR) set for accessed a
+    int taps = 0;                       // ny*nx dense, ny+nx separable
+    // folded weights: sum of the weights of every offset mapped to a rep,
+    // accumulated in fp64 and rounded once to fp32
+    float wf[kMaxTaps] = {};            // dense  [ny][nx]
+    float wyf[kMaxK] = {}, wxf[kMaxK] = {}; // separable
+};
+
+struct Candidate {
+    paraprox_scheme scheme;
+    int reach;
+    int dy, dx;
+    int taps, hy, hx, sid;
+};
+
+}  // namespace ppx
+
+struct paraprox_filter_s {
+    int ky = 1, kx = 1;
+    bool separable = false;
+    std::vector<float> w;        // dense ky*kx
+    std::vector<float> wy, wx;   // separable
+    std::mutex mu;
+    std::map<std::pair<int, int>, ppx::Plan> plans;
+};
+
+namespace ppx {
+
+// ---- plan.cpp ----
+int map_offset(int r, int d, int i);
+const Plan& get_plan(paraprox_filter f, int dy, int dx);
+void scheme_reaches(paraprox_scheme s, int reach, int* dy, int* dx);
+std::vector<Candidate> candidates(paraprox_filter f);
+
+// ---- device-side image view ----
+struct View {
+    int n, h, w;
+    long long pitch, fstride;
+    int lo, hi;  // valid input rows: [lo, hi] relative to row 0 (lo = -halo_top)
+};
+
+// ---- kernels ----
+// Each launcher enqueues on `s`, bumps the launch counter, records the kernel
+// name and returns cudaGetLastError().
+cudaError_t launch_stencil(const Plan& p, const float* in, const View& vin, float* out,
+                           long long out_pitch, long long out_fstride, cudaStream_t s);
+cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
+                           double* d_part3, double* d_scratch, cudaStream_t s);
+constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums
+
+void count_launch(const char* name);
+extern std::atomic<unsigned long long> g_launches;
+extern thread_local const char* t_last_kernel;
+
+}  // namespace ppx

@@ -1,0 +1,367 @@
+"""Thin Python binding over the libparaprox C ABI (include/paraprox.h).
+
+Argument marshalling only: every step of the path runs in the library's
+sm_100a kernels.  torch supplies device memory and the current CUDA stream.
+The names follow the C entry points without the ``paraprox_`` prefix.
+
+There is no CPU fallback: if ``libparaprox.so`` is missing this module raises
+at import, and every stencil call requires CUDA tensors.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libparaprox.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`")
+
+_lib = C.CDLL(LIB_PATH)
+
+OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CUDA, ERR_ALLOC = range(5)
+EXACT, ROW, COL, CENTER = 0, 1, 2, 3
+MRE, L2, PSNR = 0, 1, 2
+SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "column": COL, "center": CENTER, "centre": CENTER}
+SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center"}
+METRICS = {"mre": MRE, "l2": L2, "psnr": PSNR}
+MAX_K = 17
+
+
+class Image(C.Structure):
+    _fields_ = [("n", C.c_int), ("h", C.c_int), ("w", C.c_int), ("pitch", C.c_longlong),
+                ("frame_stride", C.c_longlong), ("halo_top", C.c_int), ("halo_bottom", C.c_int)]
+
+
+_P = C.c_void_p
+_I = C.POINTER(C.c_int)
+_D = C.POINTER(C.c_double)
+_F = C.POINTER(C.c_float)
+_IMG = C.POINTER(Image)
+_SIGS = {
+    "paraprox_filter_create": [C.c_int, C.c_int, _F, C.POINTER(_P)],
+    "paraprox_filter_create_separable": [C.c_int, _F, C.c_int, _F, C.POINTER(_P)],
+    "paraprox_filter_shape": [_P, _I, _I, _I],
+    "paraprox_plan_info": [_P, C.c_int, C.c_int, _I, _I, _I, _I, _I],
+    "paraprox_stencil_exact": [_P, _P, _P, _IMG, _P],
+    "paraprox_stencil_approx": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_stencil_approx_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_run_host": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_quality": [_P, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_quality_partials": [_P, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_quality_from_partials": [_D, C.c_int, _D],
+    "paraprox_tune": [_P, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
+    "paraprox_tune_candidates": [_P, C.c_int, _I, _I, _I],
+    "paraprox_tune_partials": [_P, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_tune_decide": [_P, _D, C.c_int, C.c_double, _I, _I, _D],
+}
+for _name, _args in _SIGS.items():
+    getattr(_lib, _name).argtypes = _args
+    getattr(_lib, _name).restype = C.c_int
+_lib.paraprox_filter_destroy.argtypes = [_P]
+_lib.paraprox_filter_destroy.restype = None
+_lib.paraprox_status_string.argtypes = [C.c_int]
+_lib.paraprox_status_string.restype = C.c_char_p
+_lib.paraprox_last_error.restype = C.c_char_p
+_lib.paraprox_last_kernel.restype = C.c_char_p
+_lib.paraprox_version.restype = C.c_int
+_lib.paraprox_launch_count.restype = C.c_ulonglong
+
+ABI_SYMBOLS = sorted(list(_SIGS) + ["paraprox_filter_destroy", "paraprox_status_string", "paraprox_last_error",
+                                    "paraprox_last_kernel", "paraprox_version", "paraprox_launch_count"])
+
+
+class ParaproxError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        self.status = status
+        detail = _lib.paraprox_last_error().decode()
+        super().__init__(f"{what}: {_lib.paraprox_status_string(status).decode()} ({detail})")
+
+
+def _check(rc: int, what: str):
+    if rc != OK:
+        raise ParaproxError(rc, what)
+
+
+def version() -> int:
+    return _lib.paraprox_version()
+
+
+def launch_count() -> int:
+    return int(_lib.paraprox_launch_count())
+
+
+def last_kernel() -> str:
+    return _lib.paraprox_last_kernel().decode()
+
+
+def _scheme(s) -> int:
+    if isinstance(s, str):
+        return SCHEMES[s.lower()]
+    return int(s)
+
+
+def _metric(m) -> int:
+    if isinstance(m, str):
+        return METRICS[m.lower()]
+    return int(m)
+
+
+class Filter:
+    """A filter handle (paraprox_filter_create / _separable)."""
+
+    def __init__(self, w=None, *, wy=None, wx=None):
+        h = _P()
+        if w is not None:
+            a = np.ascontiguousarray(np.asarray(w, dtype=np.float32))
+            if a.ndim == 1:
+                a = a[None]
+            if a.ndim != 2:
+                raise ValueError("dense weights must be 2-D")
+            _check(_lib.paraprox_filter_create(a.shape[0], a.shape[1], a.ctypes.data_as(_F), C.byref(h)),
+                   "filter_create")
+            self.ky, self.kx, self.separable = a.shape[0], a.shape[1], False
+        else:
+            ay = np.ascontiguousarray(np.asarray(wy, dtype=np.float32).ravel())
+            ax = np.ascontiguousarray(np.asarray(wx, dtype=np.float32).ravel())
+            _check(_lib.paraprox_filter_create_separable(ay.size, ay.ctypes.data_as(_F), ax.size,
+                                                         ax.ctypes.data_as(_F), C.byref(h)),
+                   "filter_create_separable")
+            self.ky, self.kx, self.separable = ay.size, ax.size, True
+        self._h = h
+
+    @classmethod
+    def separable_(cls, wy, wx):
+        return cls(wy=wy, wx=wx)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if self._h:
+            _lib.paraprox_filter_destroy(self._h)
+            self._h = _P()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def plan_info(self, reach_y: int, reach_x: int):
+        taps, hy, hx = C.c_int(), C.c_int(), C.c_int()
+        my = (C.c_int * self.ky)()
+        mx = (C.c_int * self.kx)()
+        _check(_lib.paraprox_plan_info(self._h, reach_y, reach_x, C.byref(taps), C.byref(hy), C.byref(hx),
+                                       my, mx), "plan_info")
+        return dict(taps=taps.value, halo_y=hy.value, halo_x=hx.value, map_y=list(my), map_x=list(mx))
+
+
+def filter_create(w) -> Filter:
+    return Filter(w)
+
+
+def filter_create_separable(wy, wx) -> Filter:
+    return Filter(wy=wy, wx=wx)
+
+
+def _stream(stream):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return C.c_void_p(stream.cuda_stream)
+
+
+def image_of(x: torch.Tensor, halo_top: int = 0, halo_bottom: int = 0) -> Image:
+    """Descriptor of a [h, w] or [n, h_total, w] fp32 tensor with unit column
+    stride; h = h_total - halo_top - halo_bottom."""
+    if x.dtype != torch.float32:
+        raise TypeError("paraprox images are fp32")
+    if x.dim() == 2:
+        n, ht, w = 1, x.shape[0], x.shape[1]
+        pitch, fs = x.stride(0), x.shape[0] * x.stride(0)
+    elif x.dim() == 3:
+        n, ht, w = x.shape
+        pitch, fs = x.stride(1), x.stride(0)
+    else:
+        raise ValueError("expected [h, w] or [n, h, w]")
+    if w > 1 and x.stride(-1) != 1:
+        raise ValueError("rows must be contiguous (unit column stride)")
+    if n > 1 and fs < ht * pitch:
+        raise ValueError("frames overlap")
+    return Image(n, ht - halo_top - halo_bottom, w, pitch, fs if n > 1 else ht * pitch, halo_top, halo_bottom)
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if not (isinstance(t, torch.Tensor) and t.is_cuda):
+            raise TypeError("paraprox device entry points take CUDA tensors (there is no CPU path)")
+
+
+def _out_like(x: torch.Tensor, halo_top: int, halo_bottom: int, out):
+    if out is not None:
+        return out
+    if x.dim() == 2:
+        return torch.empty((x.shape[0] - halo_top - halo_bottom, x.shape[1]), dtype=x.dtype, device=x.device)
+    if halo_top or halo_bottom:
+        # same pitch and frame stride as the input (the ABI shares the layout)
+        buf = torch.empty_like(x)
+        return buf[:, halo_top:x.shape[1] - halo_bottom]
+    return torch.empty_like(x)
+
+
+def _dp(t, halo_top=0):
+    return C.c_void_p(t.data_ptr() + 4 * halo_top * (t.stride(-2) if t.dim() >= 2 else 0))
+
+
+def _check_out(out, img):
+    if out.dim() == 2:
+        ok = img.n == 1 and out.shape[0] == img.h and out.shape[1] == img.w and out.stride(0) == img.pitch
+    else:
+        ok = (tuple(out.shape) == (img.n, img.h, img.w) and out.stride(1) == img.pitch
+              and (img.n == 1 or out.stride(0) == img.frame_stride))
+    if not ok or out.dtype != torch.float32 or (img.w > 1 and out.stride(-1) != 1):
+        raise ValueError("out must match the input's shape, pitch and frame stride")
+
+
+def stencil_exact(x, f: Filter, out=None, *, halo_top=0, halo_bottom=0, stream=None):
+    _need_cuda(x)
+    img = image_of(x, halo_top, halo_bottom)
+    out = _out_like(x, halo_top, halo_bottom, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_exact(f.handle, _dp(x, halo_top), _dp(out), C.byref(img), _stream(stream)),
+           "stencil_exact")
+    return out
+
+
+def stencil_approx(x, f: Filter, scheme, reach: int, out=None, *, halo_top=0, halo_bottom=0, stream=None):
+    _need_cuda(x)
+    img = image_of(x, halo_top, halo_bottom)
+    out = _out_like(x, halo_top, halo_bottom, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_approx(f.handle, _scheme(scheme), int(reach), _dp(x, halo_top), _dp(out),
+                                        C.byref(img), _stream(stream)), "stencil_approx")
+    return out
+
+
+def stencil_approx_xy(x, f: Filter, reach_y: int, reach_x: int, out=None, *, halo_top=0, halo_bottom=0,
+                      stream=None):
+    _need_cuda(x)
+    img = image_of(x, halo_top, halo_bottom)
+    out = _out_like(x, halo_top, halo_bottom, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_approx_xy(f.handle, int(reach_y), int(reach_x), _dp(x, halo_top), _dp(out),
+                                           C.byref(img), _stream(stream)), "stencil_approx_xy")
+    return out
+
+
+class Prepared:
+    """A stencil call with its arguments marshalled once (for tight loops and
+    graph capture): calling it re-issues paraprox_stencil_approx on the
+    stream given at preparation time."""
+
+    def __init__(self, x, f: Filter, scheme, reach: int, out, *, halo_top=0, halo_bottom=0, stream=None):
+        _need_cuda(x, out)
+        self._img = image_of(x, halo_top, halo_bottom)
+        _check_out(out, self._img)
+        self._keep = (x, out, f)
+        self._args = (f.handle, _scheme(scheme), int(reach), _dp(x, halo_top), _dp(out), C.byref(self._img),
+                      _stream(stream))
+        self._fn = _lib.paraprox_stencil_approx
+
+    def __call__(self):
+        rc = self._fn(*self._args)
+        if rc != OK:
+            raise ParaproxError(rc, "stencil_approx")
+
+
+def prepare(x, f: Filter, scheme, reach: int, out, **kw) -> Prepared:
+    return Prepared(x, f, scheme, reach, out, **kw)
+
+
+def run_host(x: torch.Tensor, f: Filter, scheme, reach: int, out=None, *, stream=None):
+    """End-to-end over host (ideally pinned) tensors: H2D, kernel, D2H inside
+    the library, overlapped chunk by chunk.  Returns the host output."""
+    if x.is_cuda:
+        raise TypeError("run_host takes host tensors")
+    img = image_of(x)
+    if out is None:
+        out = torch.empty_like(x, pin_memory=x.is_pinned())
+    _check_out(out, img)
+    _check(_lib.paraprox_run_host(f.handle, _scheme(scheme), int(reach), _dp(x), _dp(out), C.byref(img),
+                                  _stream(stream)), "run_host")
+    return out
+
+
+def quality(exact, approx, metric="mre", *, stream=None) -> float:
+    _need_cuda(exact, approx)
+    img = image_of(exact)
+    if exact.shape != approx.shape or exact.stride() != approx.stride():
+        raise ValueError("exact and approx must share shape and strides")
+    q = C.c_double()
+    _check(_lib.paraprox_quality(_dp(exact), _dp(approx), C.byref(img), _metric(metric), C.byref(q),
+                                 _stream(stream)), "quality")
+    return q.value
+
+
+def quality_partials(exact, approx, metric="mre", *, stream=None) -> np.ndarray:
+    _need_cuda(exact, approx)
+    img = image_of(exact)
+    if exact.shape != approx.shape or exact.stride() != approx.stride():
+        raise ValueError("exact and approx must share shape and strides")
+    p = np.zeros(3, dtype=np.float64)
+    _check(_lib.paraprox_quality_partials(_dp(exact), _dp(approx), C.byref(img), _metric(metric),
+                                          p.ctypes.data_as(_D), _stream(stream)), "quality_partials")
+    return p
+
+
+def quality_from_partials(p, metric="mre") -> float:
+    p = np.ascontiguousarray(p, dtype=np.float64)
+    q = C.c_double()
+    _check(_lib.paraprox_quality_from_partials(p.ctypes.data_as(_D), _metric(metric), C.byref(q)),
+           "quality_from_partials")
+    return q.value
+
+
+def tune_candidates(f: Filter):
+    n = C.c_int()
+    _check(_lib.paraprox_tune_candidates(f.handle, 0, C.byref(n), None, None), "tune_candidates")
+    s = (C.c_int * max(1, n.value))()
+    r = (C.c_int * max(1, n.value))()
+    _check(_lib.paraprox_tune_candidates(f.handle, n.value, C.byref(n), s, r), "tune_candidates")
+    return [(SCHEME_NAMES[s[i]], r[i]) for i in range(n.value)]
+
+
+def tune(frames, f: Filter, toq: float, metric="mre", *, stream=None):
+    """Returns (scheme name, reach, quality)."""
+    _need_cuda(frames)
+    img = image_of(frames)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune(f.handle, _dp(frames), C.byref(img), float(toq), _metric(metric), C.byref(sc),
+                              C.byref(rc), C.byref(q), _stream(stream)), "tune")
+    return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+def tune_partials(frames, f: Filter, metric="mre", *, stream=None) -> np.ndarray:
+    _need_cuda(frames)
+    img = image_of(frames)
+    n = len(tune_candidates(f))
+    p = np.zeros(3 * max(n, 1), dtype=np.float64)
+    _check(_lib.paraprox_tune_partials(f.handle, _dp(frames), C.byref(img), _metric(metric),
+                                       p.ctypes.data_as(_D), _stream(stream)), "tune_partials")
+    return p[:3 * n]
+
+
+def tune_decide(f: Filter, partials, toq: float, metric="mre"):
+    p = np.ascontiguousarray(partials, dtype=np.float64)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune_decide(f.handle, p.ctypes.data_as(_D) if p.size else None, _metric(metric),
+                                     float(toq), C.byref(sc), C.byref(rc), C.byref(q)), "tune_decide")
+    return SCHEME_NAMES[sc.value], rc.value, q.value

@@ -1,0 +1,252 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.
+
+Tolerance (reading S18): per output,
+|gpu - oracle| <= 1e-5 * sum_ij |w_ij| |X~_ij| (the oracle run on |w|, |X|),
+i.e. a 1e-5 relative error for non-negative filters, guarded against
+cancellation for signed ones.  Integer-valued decisions (the tuner) must be
+identical."""
+import numpy as np
+import pytest
+import torch
+
+import workloads as W
+from workloads import filters as F
+
+pytestmark = pytest.mark.gpu
+
+RTOL = 1e-5
+
+
+@pytest.fixture(scope="module")
+def P():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_asplos_samadijlm14_b200 as pkg
+
+    return pkg.paraprox
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+def assert_dense(P, O, x, w, dy, dx, f=None):
+    f = f or P.Filter(w)
+    g = P.stencil_approx_xy(dev(x), f, dy, dx).cpu().numpy()
+    o = O.stencil_approx_xy(x, w, dy, dx)
+    bound = RTOL * O.stencil_approx_xy(np.abs(x), np.abs(w), dy, dx) + 1e-30
+    err = np.abs(g - o)
+    assert np.all(err <= bound), (dy, dx, float((err / bound).max()), P.last_kernel())
+    return g
+
+
+def assert_sep(P, O, x, wy, wx, dy, dx, f=None):
+    f = f or P.Filter(wy=wy, wx=wx)
+    g = P.stencil_approx_xy(dev(x), f, dy, dx).cpu().numpy()
+    o = O.stencil_sep(x, wy, wx, dy, dx)
+    bound = RTOL * O.stencil_sep(np.abs(x), np.abs(wy), np.abs(wx), dy, dx) + 1e-30
+    err = np.abs(g - o)
+    assert np.all(err <= bound), (dy, dx, float((err / bound).max()), P.last_kernel())
+    return g
+
+
+DENSE = [
+    ("gauss3", F.gaussian(3)),
+    ("mean5", F.mean(5)),
+    ("conv7", F.conv(7, seed=3)),
+    ("conv9", F.conv(9)),
+    ("signed5", F.conv_signed(5)),
+    ("rect3x7", F.conv(7, seed=11, ky=3)),
+    ("rect9x1", F.conv(1, seed=12, ky=9)),
+    ("conv17", F.conv(17, seed=13)),
+    ("one", np.ones((1, 1), np.float32)),
+]
+
+
+@pytest.mark.parametrize("name,w", DENSE, ids=[d[0] for d in DENSE])
+@pytest.mark.parametrize("shape", [(2, 77, 300), (1, 257, 513)], ids=["2x77x300", "1x257x513"])
+def test_dense_all_reaches(P, O, name, w, shape):
+    """Every (dy, dx) pair, over several tiles with ragged tails."""
+    x = W.frames(*shape, seed0=1)
+    f = P.Filter(w)
+    ky, kx = w.shape
+    ry, rx = ky // 2, kx // 2
+    pairs = {(dy, dx) for dy in range(ry + 2) for dx in range(rx + 2)}
+    if len(pairs) > 40:  # 17x17: schemes x reaches only
+        pairs = {(d, d) for d in range(ry + 2)} | {(d, 0) for d in range(ry + 2)} | {(0, d) for d in range(rx + 2)}
+    for dy, dx in sorted(pairs):
+        assert_dense(P, O, x, w, dy, dx, f)
+
+
+@pytest.mark.parametrize("ky,kx", [(7, 7), (3, 5), (1, 17), (17, 1), (9, 9)])
+@pytest.mark.parametrize("shape", [(2, 77, 300), (1, 190, 700)], ids=["2x77x300", "1x190x700"])
+def test_separable_all_reaches(P, O, ky, kx, shape):
+    wy = F.conv(1, seed=40 + ky, ky=ky).ravel()
+    wx = F.conv(kx, seed=50 + kx, ky=1).ravel()
+    x = W.frames(*shape, seed0=2)
+    f = P.Filter(wy=wy, wx=wx)
+    for dy in range(ky // 2 + 2):
+        for dx in range(kx // 2 + 2):
+            assert_sep(P, O, x, wy, wx, dy, dx, f)
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 1, 1), (1, 1, 700), (1, 700, 1), (1, 5, 5), (2, 8, 8),
+                                   (1, 3, 129), (1, 33, 4), (1, 31, 127)])
+def test_degenerate_shapes(P, O, shape):
+    x = W.images.random_integers(shape, seed=3, lo=0, hi=255)
+    for w in (F.gaussian(3), F.mean(5), F.conv(9)):
+        for d in range(0, w.shape[0] // 2 + 2):
+            for dy, dx in ((d, 0), (0, d), (d, d)):
+                assert_dense(P, O, x, w, dy, dx)
+    wy, wx = F.separable(7)
+    for d in range(5):
+        assert_sep(P, O, x, wy, wx, d, d)
+
+
+@pytest.mark.parametrize("k", [3, 5, 7])
+def test_bruteforce_8x8_all_schemes(P, O, k):
+    w = F.conv(k, seed=100 + k)
+    for seed in range(3):
+        x = W.images.random_integers((8, 8), seed)
+        for scheme in ("exact", "row", "col", "center"):
+            for d in range(0, k // 2 + 2):
+                dy, dx = O.scheme_reaches(scheme, d)
+                assert_dense(P, O, x, w, dy, dx)
+
+
+def test_scheme_entry_points_agree(P, O):
+    x = W.frames(2, 70, 140, 4)
+    w = F.conv(9)
+    f = P.Filter(w)
+    xd = dev(x)
+    e = P.stencil_exact(xd, f)
+    assert torch.equal(e, P.stencil_approx(xd, f, "exact", 3))
+    assert torch.equal(e, P.stencil_approx(xd, f, "row", 0))
+    for scheme in ("row", "col", "center"):
+        for d in range(1, 6):
+            dy, dx = O.scheme_reaches(scheme, d)
+            assert torch.equal(P.stencil_approx(xd, f, scheme, d), P.stencil_approx_xy(xd, f, dy, dx))
+
+
+def test_invariants_on_gpu(P):
+    f = P.Filter(F.mean(5))
+    c = torch.full((1, 100, 200), 77.0, device="cuda")
+    for d in range(3):
+        for s in ("row", "col", "center"):
+            torch.testing.assert_close(P.stencil_approx(c, f, s, d), c, rtol=1e-6, atol=0)
+    yc = dev(np.repeat(W.image(1, 300, 5), 90, axis=0))
+    e = P.stencil_exact(yc, f)
+    for d in (1, 2):
+        torch.testing.assert_close(P.stencil_approx(yc, f, "row", d), e, rtol=2e-6, atol=0)
+
+
+def test_pitched_and_strided_layouts(P, O):
+    """pitch > w, frame_stride > h*pitch, and a misaligned base pointer."""
+    x = W.frames(3, 50, 130, 6)
+    w = F.conv(5, seed=8)
+    f = P.Filter(w)
+    o = O.stencil_exact(x, w)
+    big = torch.zeros((3, 60, 141), device="cuda")
+    big[:, 3:53, 5:135] = dev(x)
+    view = big[:, 3:53, 5:135]  # pitch 141, frame stride 60*141, offset 3*141+5 floats
+    out = torch.zeros_like(big)[:, 3:53, 5:135]
+    g = P.stencil_exact(view, f, out=out).cpu().numpy()
+    bound = RTOL * O.stencil_exact(np.abs(x), np.abs(w))
+    assert np.all(np.abs(g - o) <= bound)
+
+
+def test_stripes_with_halos_bitwise(P, O):
+    """Row stripes with halo rows reproduce the whole-image output bitwise
+    (same kernel, same tap order): the multi-GPU row-stripe decomposition."""
+    x = W.image(1000, 777, 7)
+    w = F.conv(9)
+    f = P.Filter(w)
+    xd = dev(x)
+    for dy, dx in [(0, 0), (1, 1), (4, 0), (0, 4), (2, 2)]:
+        full = P.stencil_approx_xy(xd, f, dy, dx)
+        hy = f.plan_info(dy, dx)["halo_y"]
+        for g in (2, 3, 8):
+            bounds = [1000 * k // g for k in range(g + 1)]
+            for k in range(g):
+                r0, r1 = bounds[k], bounds[k + 1]
+                ht, hb = min(hy, r0), min(hy, 1000 - r1)
+                stripe = xd[r0 - ht:r1 + hb].clone()
+                got = P.stencil_approx_xy(stripe, f, dy, dx, halo_top=ht, halo_bottom=hb)
+                assert torch.equal(got, full[r0:r1]), (dy, dx, g, k)
+
+
+def test_quality_matches_oracle_and_is_deterministic(P, O):
+    x = W.frames(3, 300, 400, 9)
+    f = P.Filter(F.mean(5))
+    xd = dev(x)
+    e = P.stencil_exact(xd, f)
+    a = P.stencil_approx(xd, f, "center", 1)
+    en, an = e.cpu().numpy().astype(np.float64), a.cpu().numpy().astype(np.float64)
+    for m in ("mre", "l2", "psnr"):
+        q1 = P.quality(e, a, m)
+        q2 = P.quality(e, a, m)
+        assert q1 == q2
+        qo = O.quality(en, an, m)
+        assert abs(q1 - qo) <= 1e-12 * max(1.0, abs(qo)), (m, q1, qo)
+    assert P.quality(e, e, "mre") == 1.0
+    # partials add across disjoint pixel sets
+    p0 = P.quality_partials(e[:1], a[:1], "l2")
+    p1 = P.quality_partials(e[1:], a[1:], "l2")
+    assert P.quality_from_partials(p0 + p1, "l2") == pytest.approx(P.quality(e, a, "l2"), abs=1e-14)
+
+
+TUNE_CASES = [
+    ("gauss3", F.gaussian(3), "mre", (10, 256, 256)),
+    ("mean5", F.mean(5), "mre", (10, 256, 256)),
+    ("conv9", F.conv(9), "l2", (10, 256, 256)),
+    ("sep7", F.separable(7), "l2", (10, 216, 384)),
+]
+
+
+@pytest.mark.parametrize("name,w,metric,shape", TUNE_CASES, ids=[t[0] for t in TUNE_CASES])
+def test_tuner_bit_identical(P, O, name, w, metric, shape):
+    x = W.frames(*shape, seed0=0)
+    f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+    xd = dev(x)
+    parts = P.tune_partials(xd, f, metric)
+    ref_all = O.tune(x, w, 2.0 if metric != "psnr" else 1e9, metric, all_qualities=True)["qualities"]
+    qs = [P.quality_from_partials(parts[3 * k:3 * k + 3], metric) for k in range(len(ref_all))]
+    np.testing.assert_allclose(qs, ref_all, rtol=0, atol=1e-7)
+    for toq in (0.80, 0.90, 0.95, 0.99):
+        got = P.tune(xd, f, toq, metric)
+        ref = O.tune(x, w, toq, metric)
+        margin = min(abs(q - toq) for q in ref_all)
+        assert got[:2] == (ref["scheme"], ref["reach"]), (toq, got, ref, margin)
+        assert P.tune_decide(f, parts, toq, metric) == got
+        print(f"{name} toq={toq}: {got[0]}:{got[1]} q={got[2]:.6f} (oracle {ref['quality']:.6f}), "
+              f"min |q-toq| = {margin:.2e}")
+
+
+def test_tuner_tpins_on_gpu(P):
+    f = P.Filter(F.mean(5))
+    yc = dev(np.repeat(W.image(1, 128, 3), 64, axis=0)[None])
+    assert P.tune(yc, f, 1 - 1e-6, "mre")[:2] == ("row", 2)
+    const = torch.full((2, 64, 64), 120.0, device="cuda")
+    assert P.tune(const, f, 1 - 1e-6, "l2")[:2] == ("center", 2)
+    noise = dev(W.uniform_noise(128, 128, 5)[None])
+    assert P.tune(noise, f, 0.95, "mre") == ("exact", 0, 1.0)
+
+
+def test_run_host_matches_device_path(P):
+    for shape, w in [((1, 1500, 900), F.conv(9)), ((5, 120, 256), F.mean(5))]:
+        x = torch.from_numpy(W.frames(*shape, seed0=12)).pin_memory()
+        f = P.Filter(w)
+        for scheme, d in [("exact", 0), ("row", 1), ("center", 2)]:
+            host = P.run_host(x[0] if shape[0] == 1 else x, f, scheme, d)
+            ref = P.stencil_approx(x.cuda(), f, scheme, d).cpu()
+            assert torch.equal(host, ref[0] if shape[0] == 1 else ref), (shape, scheme, d)
+
+
+def test_launches_counted(P):
+    f = P.Filter(F.gaussian(3))
+    x = torch.rand(1, 64, 64, device="cuda")
+    n0 = P.launch_count()
+    P.stencil_exact(x, f)
+    P.stencil_approx(x, f, "row", 1)
+    torch.cuda.synchronize()
+    assert P.launch_count() - n0 == 2
