@@ -140,7 +140,7 @@ def oracle_run(x, kind, w, scheme, reach):
     return oracle.stencil_approx(x, w, scheme, reach)
 
 
-def cpu_baseline(wl, kind, w, scheme, reach, budget_s=12.0, max_reps=16):
+def cpu_baseline(wl, kind, w, scheme, reach, budget_s=10.0, max_reps=400):
     """The oracle as it stands, on the host cores, over a bounded sample of the
     workload: whole frames (or a row band of the c4 image) until ~budget_s."""
     import oracle

@@ -1,13 +1,153 @@
 // dispatch.cu -- picks the kernel variant for a plan and an image layout.
-#include "internal.h"
+//
+// Fast path: the persistent TMA tile kernel instance (k_tiles.cuh) whose
+// compile-time accessed-offset masks equal the plan's (every plan of a filter
+// up to 9x9 has one; instances are registered by inst_r*_*.cu).  It needs a
+// layout TMA can describe (16-byte aligned rows) and 16-byte aligned output
+// rows.  Anything else takes the generic kernel (k_generic.cu): slower, same
+// results, still on the GPU.
+#include <cstdlib>
+#include <mutex>
+#include <vector>
+
+#include "k_tiles.cuh"
 
 namespace ppx {
 
 cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float* out, long long opitch,
                            long long ofs, cudaStream_t s);
 
+void register_r1_dense();
+void register_r2_dense();
+void register_r3_dense();
+void register_r4_dense();
+void register_r1_sep();
+void register_r2_sep();
+void register_r3_sep();
+void register_r4_sep();
+
+namespace {
+
+constexpr int kMaxDev = 64;
+
+struct Entry {
+    TileInstance ti;
+    bool ready[kMaxDev] = {};
+    int occ[kMaxDev] = {};
+};
+
+std::vector<Entry>& reg() {
+    static std::vector<Entry> r;
+    return r;
+}
+
+std::mutex g_mu;
+int g_sms[kMaxDev] = {};
+
+void init_registry() {
+    static std::once_flag once;
+    std::call_once(once, [] {
+        register_r1_dense();
+        register_r2_dense();
+        register_r3_dense();
+        register_r4_dense();
+        register_r1_sep();
+        register_r2_sep();
+        register_r3_sep();
+        register_r4_sep();
+    });
+}
+
+bool force_generic() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("PARAPROX_FORCE_GENERIC");
+        v = (e && e[0] == '1') ? 1 : 0;
+    }
+    return v == 1;
+}
+
+}  // namespace
+
+void register_tile_instance(const TileInstance& ti) {
+    Entry e;
+    e.ti = ti;
+    reg().push_back(e);
+}
+
+static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const View& v, float* out,
+                                long long opitch, long long ofs, cudaStream_t s, bool* taken) {
+    *taken = false;
+    int dev = 0;
+    cudaError_t err = cudaGetDevice(&dev);
+    if (err != cudaSuccess) return err;
+    if (dev >= kMaxDev) return cudaSuccess;
+    // layout checks: TMA-describable input, 16-byte aligned output rows
+    if ((reinterpret_cast<uintptr_t>(out) & 15) || (opitch & 3) || (v.n > 1 && (ofs & 3))) return cudaSuccess;
+    const int rows_valid = v.hi - v.lo + 1;
+    const long long fstride = v.n > 1 ? v.fstride : (long long)rows_valid * v.pitch;
+    CUtensorMap tmap;
+    const int box_w = kTW + 2 * round4(e.ti.hx), box_h = kTH + 2 * e.ti.hy;
+    if (!encode_tmap_3d(&tmap, in + (long long)v.lo * v.pitch, v.w, rows_valid, v.n, v.pitch, fstride, box_w, box_h))
+        return cudaSuccess;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        if (!e.ready[dev]) {
+            err = cudaFuncSetAttribute(e.ti.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, e.ti.smem);
+            if (err != cudaSuccess) return err;
+            int occ = 0;
+            err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, e.ti.fn, kThreads, e.ti.smem);
+            if (err != cudaSuccess) return err;
+            if (!g_sms[dev]) {
+                err = cudaDeviceGetAttribute(&g_sms[dev], cudaDevAttrMultiProcessorCount, dev);
+                if (err != cudaSuccess) return err;
+            }
+            e.occ[dev] = occ > 0 ? occ : 1;
+            e.ready[dev] = true;
+        }
+    }
+    TileArgs A;
+    A.n = v.n;
+    A.h = v.h;
+    A.w = v.w;
+    A.rows_valid = rows_valid;
+    A.row_off = -v.lo;
+    A.tiles_x = (v.w + kTW - 1) / kTW;
+    A.tiles_y = (v.h + kTH - 1) / kTH;
+    const long long nt = (long long)A.tiles_x * A.tiles_y * v.n;
+    if (nt >= (1LL << 31)) return cudaSuccess;
+    A.ntiles = (int)nt;
+    A.out = out;
+    A.opitch = opitch;
+    A.ofs = ofs;
+    TapW W = {};
+    if (p.separable) {
+        for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 4] = p.wyf[i];
+        for (int j = 0; j < p.nx; ++j) W.wx[p.ax[j] + 4] = p.wxf[j];
+    } else {
+        for (int i = 0; i < p.ny; ++i)
+            for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];
+    }
+    const long long cap = (long long)g_sms[dev] * e.occ[dev];
+    const int grid = (int)(nt < cap ? nt : cap);
+    e.ti.fn<<<grid, kThreads, e.ti.smem, s>>>(tmap, A, W);
+    count_launch(e.ti.name);
+    *taken = true;
+    return cudaGetLastError();
+}
+
 cudaError_t launch_stencil(const Plan& p, const float* in, const View& v, float* out, long long opitch,
                            long long ofs, cudaStream_t s) {
+    if (!force_generic() && p.ry <= 4 && p.rx <= 4) {
+        init_registry();
+        for (Entry& e : reg()) {
+            if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;
+            bool taken = false;
+            cudaError_t err = launch_tiles(e, p, in, v, out, opitch, ofs, s, &taken);
+            if (err != cudaSuccess || taken) return err;
+            break;
+        }
+    }
     return launch_generic(p, in, v, out, opitch, ofs, s);
 }
 

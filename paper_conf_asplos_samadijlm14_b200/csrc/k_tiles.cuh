@@ -1,0 +1,291 @@
+// k_tiles.cuh -- the fast stencil kernels (dense and fused separable), one
+// template over the approximation's accessed offsets.
+//
+// Design:
+//  * Persistent CTAs (grid = resident CTAs, <= #SMs x occupancy) walk output
+//    tiles of TH x TW = 64 x 128 in raster order (frame, tile row, tile col),
+//    so concurrently running CTAs share their halo rows in L2.
+//  * A STAGES-deep ring of shared-memory tiles filled by TMA
+//    (cp.async.bulk.tensor.3d, mbarrier complete_tx): the (TH + 2HY) x
+//    (TW + 2HXP) input box of tile i+STAGES-1 streams in while tile i is
+//    computed.  Only the halo the *approximation* needs is staged: HY/HX are
+//    the largest accessed offsets (the reaching distance shrinks them, e.g.
+//    the row scheme at full reach stages no halo rows at all).
+//  * Clamp-to-edge: TMA zero-fills out-of-range boxes; rows are clamped at
+//    read time (the smem row index is clamped to the valid rows) and border
+//    columns are replicated in shared memory before the compute.
+//  * Register blocking: a thread owns RB = 8 rows x 4 columns of outputs; it
+//    streams the staged rows once (128-bit LDS, conflict-free) and applies
+//    each row to every output row it contributes to.  Only the accessed
+//    offsets (bit masks MASKY / MASKX, compile-time) generate FMAs: the
+//    folded weights of the plan (plan.cpp) sit in the kernel parameter bank.
+//  * Separable filters: horizontal pass on the staged rows (results written
+//    back in place), then the vertical pass -- one HBM read and one write per
+//    pixel for both passes.
+//  * Outputs leave as 128-bit streaming stores (st.global.cs).
+#pragma once
+
+#include "internal.h"
+#include "tma.cuh"
+
+namespace ppx {
+
+constexpr int kTW = 128;                 // tile width (outputs)
+constexpr int kRB = 8;                   // output rows per thread
+constexpr int kWarps = 8;                // 256 threads
+constexpr int kTH = kRB * kWarps;        // 64 tile rows
+constexpr int kThreads = 32 * kWarps;
+
+struct TapW {
+    float w[9][9];   // dense folded weights at [a + 4][b + 4]
+    float wy[9];     // separable folded weights at [a + 4]
+    float wx[9];
+};
+
+struct TileArgs {
+    int n, h, w;
+    int rows_valid;  // valid input rows per frame (descriptor rows)
+    int row_off;     // descriptor row of output row 0 (= halo_top)
+    int tiles_x, tiles_y, ntiles;
+    float* out;
+    long long opitch, ofs;
+};
+
+__host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
+
+template <int HY, int HX>
+struct Geom {
+    static constexpr int HXP = round4(HX);
+    static constexpr int SW = kTW + 2 * HXP;   // staged row length (floats)
+    static constexpr int SH = kTH + 2 * HY;    // staged rows
+    static constexpr int STAGE_BYTES = SW * SH * 4;
+    static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
+    static constexpr int STAGES = (3 * STAGE_STRIDE <= 110 * 1024) ? 3 : 2;
+    static constexpr int SMEM = STAGES * STAGE_STRIDE;
+};
+
+__device__ __forceinline__ constexpr bool has(uint32_t mask, int off) { return (mask >> (off + 8)) & 1u; }
+
+// does staged row rr (relative to the thread's first output row) feed any of
+// the thread's RB output rows?
+template <uint32_t MASKY, int HY>
+__device__ __forceinline__ constexpr bool row_needed(int rr) {
+    for (int k = 0; k < kRB; ++k) {
+        const int a = rr - HY - k;
+        if (a >= -HY && a <= HY && has(MASKY, a)) return true;
+    }
+    return false;
+}
+
+template <int NV>
+__device__ __forceinline__ void load_row(const float* row, int lane, float (&v)[NV]) {
+    const float4* p = reinterpret_cast<const float4*>(row) + lane;
+#pragma unroll
+    for (int q = 0; q < NV / 4; ++q) {
+        const float4 t = p[q];
+        v[4 * q + 0] = t.x;
+        v[4 * q + 1] = t.y;
+        v[4 * q + 2] = t.z;
+        v[4 * q + 3] = t.w;
+    }
+}
+
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+__global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ CUtensorMap tmap,
+                                                       const TileArgs A, const __grid_constant__ TapW W) {
+    using G = Geom<HY, HX>;
+    constexpr int HXP = G::HXP, SW = G::SW, SH = G::SH, NV = 4 + 2 * HXP;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ uint64_t bars[G::STAGES];
+
+    const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
+    const int tiles_per_frame = A.tiles_x * A.tiles_y;
+
+    auto coords = [&](int t, int& f, int& y0, int& x0) {
+        f = t / tiles_per_frame;
+        const int r = t - f * tiles_per_frame;
+        const int ty = r / A.tiles_x;
+        y0 = ty * kTH;
+        x0 = (r - ty * A.tiles_x) * kTW;
+    };
+    auto issue = [&](int t, int s) {
+        int f, y0, x0;
+        coords(t, f, y0, x0);
+        fence_proxy_async();
+        mbar_expect_tx(&bars[s], G::STAGE_BYTES);
+        tma_load_3d(smem_raw + s * G::STAGE_STRIDE, &tmap, x0 - HXP, y0 + A.row_off - HY, f, &bars[s]);
+    };
+
+    if (tid == 0) {
+        for (int s = 0; s < G::STAGES; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+        tma_prefetch_desc(&tmap);
+    }
+    __syncthreads();
+    if (tid == 0)
+        for (int s = 0; s < G::STAGES - 1; ++s) {
+            const int t = blockIdx.x + s * gridDim.x;
+            if (t < A.ntiles) issue(t, s);
+        }
+
+    int it = 0;
+    for (int tile = blockIdx.x; tile < A.ntiles; tile += gridDim.x, ++it) {
+        const int s = it % G::STAGES;
+        if (tid == 0) {
+            const int ahead = tile + (G::STAGES - 1) * gridDim.x;
+            if (ahead < A.ntiles) issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+        }
+        int f, y0, x0;
+        coords(tile, f, y0, x0);
+        float* S = reinterpret_cast<float*>(smem_raw + s * G::STAGE_STRIDE);
+        mbar_wait(&bars[s], (it / G::STAGES) & 1);
+
+        // valid staged rows / columns of this tile
+        const int drow0 = y0 + A.row_off - HY;
+        const int rlo = max(0, -drow0);
+        const int rhi = min(SH - 1, A.rows_valid - 1 - drow0);
+        const int clo = max(0, HXP - x0);
+        const int chi = min(SW - 1, A.w - 1 - x0 + HXP);
+        if (clo > 0 || chi < SW - 1) {  // border columns: replicate the edge (clamp)
+            for (int idx = tid; idx < SH * SW; idx += kThreads) {
+                const int r = idx / SW, c = idx - r * SW;
+                if (c < clo) S[r * SW + c] = S[r * SW + clo];
+                else if (c > chi) S[r * SW + c] = S[r * SW + chi];
+            }
+            __syncthreads();
+        }
+
+        const int ty0 = wi * kRB;
+        float acc[kRB][4];
+#pragma unroll
+        for (int k = 0; k < kRB; ++k) acc[k][0] = acc[k][1] = acc[k][2] = acc[k][3] = 0.f;
+
+        if constexpr (!SEP) {
+#pragma unroll
+            for (int rr = 0; rr < kRB + 2 * HY; ++rr) {
+                if (!row_needed<MASKY, HY>(rr)) continue;
+                const int sr = min(max(ty0 + rr, rlo), rhi);
+                float v[NV];
+                load_row<NV>(S + sr * SW, lane, v);
+#pragma unroll
+                for (int k = 0; k < kRB; ++k) {
+                    const int a = rr - HY - k;
+                    if (a < -HY || a > HY || !has(MASKY, a)) continue;
+#pragma unroll
+                    for (int b = -HX; b <= HX; ++b) {
+                        if (!has(MASKX, b)) continue;
+                        const float wt = W.w[a + 4][b + 4];
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) acc[k][c] = fmaf(wt, v[HXP + c + b], acc[k][c]);
+                    }
+                }
+            }
+        } else {
+            // horizontal pass over the staged rows (clamped), kept in registers
+            constexpr int RPT = (SH + kWarps - 1) / kWarps;  // rows per thread
+            float hz[RPT][4];
+#pragma unroll
+            for (int q = 0; q < RPT; ++q) {
+                const int r = wi + q * kWarps;
+                if (r < SH) {
+                    const int sr = min(max(r, rlo), rhi);
+                    float v[NV];
+                    load_row<NV>(S + sr * SW, lane, v);
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) hz[q][c] = 0.f;
+#pragma unroll
+                    for (int b = -HX; b <= HX; ++b) {
+                        if (!has(MASKX, b)) continue;
+                        const float wt = W.wx[b + 4];
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) hz[q][c] = fmaf(wt, v[HXP + c + b], hz[q][c]);
+                    }
+                }
+            }
+            __syncthreads();  // every thread has read its rows: overwrite in place
+#pragma unroll
+            for (int q = 0; q < RPT; ++q) {
+                const int r = wi + q * kWarps;
+                if (r < SH)
+                    reinterpret_cast<float4*>(S + r * SW + HXP)[lane] = make_float4(hz[q][0], hz[q][1], hz[q][2], hz[q][3]);
+            }
+            __syncthreads();
+            // vertical pass (rows already clamped by the horizontal pass)
+#pragma unroll
+            for (int rr = 0; rr < kRB + 2 * HY; ++rr) {
+                if (!row_needed<MASKY, HY>(rr)) continue;
+                const float4 t = reinterpret_cast<const float4*>(S + (ty0 + rr) * SW + HXP)[lane];
+#pragma unroll
+                for (int k = 0; k < kRB; ++k) {
+                    const int a = rr - HY - k;
+                    if (a < -HY || a > HY || !has(MASKY, a)) continue;
+                    const float wt = W.wy[a + 4];
+                    acc[k][0] = fmaf(wt, t.x, acc[k][0]);
+                    acc[k][1] = fmaf(wt, t.y, acc[k][1]);
+                    acc[k][2] = fmaf(wt, t.z, acc[k][2]);
+                    acc[k][3] = fmaf(wt, t.w, acc[k][3]);
+                }
+            }
+        }
+
+        // stores: 128-bit streaming where the 4 columns are inside the image
+        const int x = x0 + 4 * lane;
+        float* obase = A.out + (long long)f * A.ofs + x;
+#pragma unroll
+        for (int k = 0; k < kRB; ++k) {
+            const int y = y0 + ty0 + k;
+            if (y < A.h && x < A.w) {
+                float* o = obase + (long long)y * A.opitch;
+                if (x + 3 < A.w) {
+                    __stcs(reinterpret_cast<float4*>(o), make_float4(acc[k][0], acc[k][1], acc[k][2], acc[k][3]));
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (x + c < A.w) __stcs(o + c, acc[k][c]);
+                }
+            }
+        }
+        __syncthreads();  // stage s fully consumed before it is refilled
+    }
+}
+
+// ---- registry -----------------------------------------------------------
+
+using TileKernel = void (*)(const CUtensorMap, const TileArgs, const TapW);
+
+struct TileInstance {
+    bool sep;
+    uint32_t masky, maskx;
+    int hy, hx;
+    TileKernel fn;
+    int smem;
+    const char* name;
+};
+
+void register_tile_instance(const TileInstance& ti);
+
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+TileInstance make_instance(const char* name) {
+    TileInstance ti;
+    ti.sep = SEP;
+    ti.masky = MASKY;
+    ti.maskx = MASKX;
+    ti.hy = HY;
+    ti.hx = HX;
+    ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP>;
+    ti.smem = Geom<HY, HX>::SMEM;
+    ti.name = name;
+    return ti;
+}
+
+// rep-offset sets that occur for radii <= 4 (bit a + 8 per accessed offset a)
+#define PPX_S0 (1u << 8)                                  /* {0}           */
+#define PPX_F1 (0x7u << 7)                                /* {-1..1}       */
+#define PPX_F2 (0x1Fu << 6)                               /* {-2..2}       */
+#define PPX_F3 (0x7Fu << 5)                               /* {-3..3}       */
+#define PPX_F4 (0x1FFu << 4)                              /* {-4..4}       */
+#define PPX_L2 ((1u << 6) | (1u << 8) | (1u << 10))       /* {-2, 0, 2}    */
+#define PPX_L3 ((1u << 5) | (1u << 8) | (1u << 11))       /* {-3, 0, 3}    */
+#define PPX_L4 ((1u << 4) | (1u << 8) | (1u << 12))       /* {-4, 0, 4}    */
+
+}  // namespace ppx

@@ -250,3 +250,36 @@ def test_launches_counted(P):
     P.stencil_approx(x, f, "row", 1)
     torch.cuda.synchronize()
     assert P.launch_count() - n0 == 2
+
+
+@pytest.mark.parametrize("kind,w", [("dense", F.gaussian(3)), ("dense", F.mean(5)), ("dense", F.conv(9)),
+                                    ("dense", F.conv(7, seed=3)), ("sep", F.separable(7))])
+def test_fast_path_taken(P, kind, w):
+    """Aligned layouts of every BASELINE filter take the TMA tile kernels."""
+    f = P.Filter(wy=w[0], wx=w[1]) if kind == "sep" else P.Filter(w)
+    x = torch.rand(2, 200, 260, device="cuda")
+    r = f.ky // 2
+    for dy, dx in [(0, 0), (r, r), (1, 0), (0, 1), (r, 0), (0, r)]:
+        P.stencil_approx_xy(x, f, dy, dx)
+        assert P.last_kernel().startswith(kind + "_"), (dy, dx, P.last_kernel())
+
+
+@pytest.mark.parametrize("w", [F.mean(5), F.conv(9), F.conv_signed(5), F.gaussian(3)])
+def test_generic_and_tile_kernels_bitwise(P, w):
+    """The tile kernel and the generic kernel sum the folded taps in the same
+    order: an aligned (tile path) and a misaligned (generic path) copy of the
+    same image give identical bits."""
+    f = P.Filter(w)
+    x = dev(W.frames(2, 150, 333, 30))
+    buf = torch.zeros(2 * 150 * 333 + 1, device="cuda")
+    mis = buf[1:].view(2, 150, 333)
+    mis.copy_(x)
+    r = w.shape[0] // 2
+    for dy, dx in [(0, 0), (1, 1), (r, 0), (0, r), (r, r)]:
+        a = P.stencil_approx_xy(x, f, dy, dx)
+        ka = P.last_kernel()
+        ob = torch.zeros(2 * 150 * 333 + 1, device="cuda")[1:].view(2, 150, 333)
+        b = P.stencil_approx_xy(mis, f, dy, dx, out=ob)
+        kb = P.last_kernel()
+        assert ka != "generic" and kb == "generic", (ka, kb)
+        assert torch.equal(a, b), (dy, dx)
