@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstring>
 #include <new>
+#include <mutex>
 #include <string>
 
 #include "internal.h"
@@ -104,7 +105,32 @@ static double quality_of(const double* p3, paraprox_metric m) {
 
 static bool metric_ok(paraprox_metric m) { return m == PARAPROX_MRE || m == PARAPROX_L2 || m == PARAPROX_PSNR; }
 
-// scratch for one quality reduction: 2*kQualityBlocks partials + 3 results
+// Stream-ordered scratch comes from a library-owned memory pool per device
+// whose release threshold keeps freed blocks mapped, so repeated calls (the
+// tuner, run_host) do not remap device memory every time.
+static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev >= 64) return cudaMallocAsync(p, bytes, s);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        if (!pools[dev]) {
+            cudaMemPoolProps props = {};
+            props.allocType = cudaMemAllocationTypePinned;
+            props.location.type = cudaMemLocationTypeDevice;
+            props.location.id = dev;
+            e = cudaMemPoolCreate(&pools[dev], &props);
+            if (e != cudaSuccess) return e;
+            uint64_t keep = ~0ull;
+            cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &keep);
+        }
+    }
+    return cudaMallocFromPoolAsync(p, bytes, pools[dev], s);
+}
+
 struct DevBuf {
     void* p = nullptr;
     cudaStream_t s = nullptr;
@@ -122,7 +148,7 @@ static paraprox_status quality_partials_impl(const float* e, const float* a, con
     cudaStream_t cs = (cudaStream_t)s;
     DevBuf buf;
     buf.s = cs;
-    PPX_CUDA(cudaMallocAsync(&buf.p, sizeof(double) * (2 * kQualityBlocks + 3), cs));
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * (2 * kQualityBlocks + 3), cs));
     double* d = (double*)buf.p;
     cudaError_t err = launch_quality(e, a, view_of(img), m, d + 2 * kQualityBlocks, d, cs);
     if (err != cudaSuccess) return cuda_fail(err, "quality launch");
@@ -147,7 +173,7 @@ static paraprox_status tune_partials_impl(paraprox_filter f, const float* d_trai
     DevBuf buf;
     buf.s = cs;
     const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (2 * kQualityBlocks + 3 * nc) + 256;
-    PPX_CUDA(cudaMallocAsync(&buf.p, bytes, cs));
+    PPX_CUDA(scratch_alloc(&buf.p, bytes, cs));
     float* E = (float*)buf.p;
     float* A = E + count;
     double* scratch = (double*)(((uintptr_t)(A + count) + 255) & ~(uintptr_t)255);
@@ -357,7 +383,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     const long long hfs = n > 1 ? img->frame_stride : 0;
     DevBuf buf;
     buf.s = cs;
-    PPX_CUDA(cudaMallocAsync(&buf.p, sizeof(float) * 2 * plane * n, cs));
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(float) * 2 * plane * n, cs));
     float* din = (float*)buf.p;
     float* dout = din + plane * n;
     // chunks: frames when batched, else row bands (halo rows come along)

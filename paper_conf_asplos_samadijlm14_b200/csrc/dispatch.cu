@@ -130,7 +130,18 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     }
     const long long cap = (long long)g_sms[dev] * e.occ[dev];
     const int grid = (int)(nt < cap ? nt : cap);
-    e.ti.fn<<<grid, kThreads, e.ti.smem, s>>>(tmap, A, W);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = e.ti.smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    err = cudaLaunchKernelEx(&cfg, e.ti.fn, tmap, A, W);
+    if (err != cudaSuccess) return err;
     count_launch(e.ti.name);
     *taken = true;
     return cudaGetLastError();

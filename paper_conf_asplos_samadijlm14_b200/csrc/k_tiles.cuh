@@ -122,6 +122,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         tma_prefetch_desc(&tmap);
     }
     __syncthreads();
+    // Programmatic dependent launch: the prologue above overlapped the tail of
+    // the previous kernel in the stream; no global memory is touched before
+    // the previous grid has completed and flushed.  Our own dependents may be
+    // scheduled as soon as SMs free up.
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s) {
             const int t = blockIdx.x + s * gridDim.x;

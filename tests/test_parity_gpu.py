@@ -270,15 +270,15 @@ def test_generic_and_tile_kernels_bitwise(P, w):
     order: an aligned (tile path) and a misaligned (generic path) copy of the
     same image give identical bits."""
     f = P.Filter(w)
-    x = dev(W.frames(2, 150, 333, 30))
-    buf = torch.zeros(2 * 150 * 333 + 1, device="cuda")
-    mis = buf[1:].view(2, 150, 333)
+    x = dev(W.frames(2, 150, 336, 30))
+    buf = torch.zeros(2 * 150 * 336 + 1, device="cuda")
+    mis = buf[1:].view(2, 150, 336)
     mis.copy_(x)
     r = w.shape[0] // 2
     for dy, dx in [(0, 0), (1, 1), (r, 0), (0, r), (r, r)]:
         a = P.stencil_approx_xy(x, f, dy, dx)
         ka = P.last_kernel()
-        ob = torch.zeros(2 * 150 * 333 + 1, device="cuda")[1:].view(2, 150, 333)
+        ob = torch.zeros(2 * 150 * 336 + 1, device="cuda")[1:].view(2, 150, 336)
         b = P.stencil_approx_xy(mis, f, dy, dx, out=ob)
         kb = P.last_kernel()
         assert ka != "generic" and kb == "generic", (ka, kb)
