@@ -70,6 +70,8 @@ bool force_generic() {
 }  // namespace
 
 void register_tile_instance(const TileInstance& ti) {
+    for (const Entry& o : reg())  // the same instance serves several radii
+        if (o.ti.fn == ti.fn) return;
     Entry e;
     e.ti = ti;
     reg().push_back(e);
