@@ -1,0 +1,166 @@
+"""Multi-GPU orchestration of the stencil hot path (DESIGN.md
+"Multi-GPU").  One process per GPU, torch.distributed (NCCL over NVLink /
+NVSwitch) for the plumbing.  The paper is single-device; the decompositions
+below are this build's.
+
+* P1 frame sharding: independent frames split across ranks, no data-path
+  collective (``frame_shard``).  Pooled tuning / quality all-reduce three fp64
+  partial sums per candidate (``tune_pooled``, ``quality_pooled``), so every
+  rank reaches the identical decision with no broadcast.
+* P2 row stripes of one large image: rank k owns rows [r0, r1) and keeps
+  ``halo`` rows above and below; one halo exchange per step with the two
+  neighbours (``exchange_halos``, batch_isend_irecv) overlapped with the
+  interior rows, then the two boundary bands (``stencil_stripe``).  The
+  approximation shrinks the halo to the largest accessed row offset h_y; the
+  row and centre schemes at full reach have h_y = 0 and need no exchange.
+  Edge ranks clamp at the true image edge (halo_top / halo_bottom = 0).
+
+All compute goes through the C ABI binding (``paraprox``); the ``compute``
+hook of ``stencil_stripe`` exists only so the exchange logic can be tested on
+CPU with the gloo backend against the oracle (tests/test_dist_gloo.py).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+
+def frame_shard(n: int, world: int, rank: int):
+    """Frames [f0, f1) of rank `rank` (contiguous, sizes differ by <= 1)."""
+    f0 = n * rank // world
+    f1 = n * (rank + 1) // world
+    return f0, f1
+
+
+@dataclass
+class Stripe:
+    r0: int          # first owned row (global)
+    r1: int          # one past the last owned row
+    cap: int         # halo capacity allocated above and below
+    h: int           # global image rows
+
+    @property
+    def rows(self) -> int:
+        return self.r1 - self.r0
+
+    def halo_top(self, hy: int) -> int:
+        """Valid halo rows above the stripe for a plan with halo hy."""
+        return min(hy, self.r0)
+
+    def halo_bottom(self, hy: int) -> int:
+        return min(hy, self.h - self.r1)
+
+
+def stripe_of(h: int, world: int, rank: int, cap: int) -> Stripe:
+    r0 = h * rank // world
+    r1 = h * (rank + 1) // world
+    return Stripe(r0, r1, cap, h)
+
+
+def alloc_stripe(s: Stripe, w: int, device=None, dtype=torch.float32) -> torch.Tensor:
+    """[cap + rows + cap, w] buffer; owned rows at [cap, cap + rows)."""
+    return torch.empty((s.cap + s.rows + s.cap, w), dtype=dtype, device=device)
+
+
+def exchange_halos(buf: torch.Tensor, s: Stripe, hy: int, group=None, async_op: bool = False):
+    """Send the top hy owned rows to rank-1 and the bottom hy owned rows to
+    rank+1; receive their boundary rows into this stripe's halos.  Rows are
+    contiguous, so every message is one contiguous tensor (no pack kernel).
+    Returns the list of requests (async_op) or waits for them."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    if hy <= 0 or world == 1:
+        return []
+    if hy > s.cap:
+        raise ValueError("halo larger than the allocated capacity")
+    if s.rows < hy:
+        raise ValueError("stripe thinner than the halo")
+    ops = []
+    c, n = s.cap, s.rows
+    if rank > 0:
+        peer = dist.get_global_rank(group, rank - 1) if group is not None else rank - 1
+        ops.append(dist.P2POp(dist.isend, buf[c:c + hy], peer, group))
+        ops.append(dist.P2POp(dist.irecv, buf[c - hy:c], peer, group))
+    if rank < world - 1:
+        peer = dist.get_global_rank(group, rank + 1) if group is not None else rank + 1
+        ops.append(dist.P2POp(dist.isend, buf[c + n - hy:c + n], peer, group))
+        ops.append(dist.P2POp(dist.irecv, buf[c + n:c + n + hy], peer, group))
+    reqs = dist.batch_isend_irecv(ops)
+    if async_op:
+        return reqs
+    for r in reqs:
+        r.wait()
+    return []
+
+
+def _band(buf, s: Stripe, y0: int, y1: int, top: int, bottom: int):
+    """View of owned rows [y0, y1) with `top` valid rows above and `bottom`
+    below, as (tensor including halos, halo_top, halo_bottom)."""
+    c = s.cap
+    return buf[c + y0 - top:c + y1 + bottom], top, bottom
+
+
+def stencil_stripe(buf: torch.Tensor, s: Stripe, f, scheme, reach: int, out: torch.Tensor,
+                   group=None, compute=None, hy: int | None = None):
+    """One row-stripe step: halo exchange overlapped with the interior rows,
+    then the boundary bands.  `out` is [rows, w].  `compute(band, ht, hb,
+    out_rows)` defaults to the CUDA stencil through the C ABI."""
+    if compute is None:
+        from . import paraprox as P
+
+        def compute(band, ht, hb, o):
+            P.stencil_approx(band, f, scheme, reach, out=o, halo_top=ht, halo_bottom=hb)
+    if hy is None:
+        dy = {"exact": 0, "row": reach, "col": 0, "center": reach, "centre": reach}[scheme]
+        dx = {"exact": 0, "row": 0, "col": reach, "center": reach, "centre": reach}[scheme]
+        hy = f.plan_info(dy, dx)["halo_y"]
+    n = s.rows
+    ht, hb = s.halo_top(hy), s.halo_bottom(hy)
+    if hy == 0 or n <= 2 * hy:
+        exchange_halos(buf, s, hy, group)
+        band, t, b = _band(buf, s, 0, n, ht, hb)
+        compute(band, t, b, out)
+        return out
+    reqs = exchange_halos(buf, s, hy, group, async_op=True)
+    # interior rows [hy, n - hy): every input row they read is owned
+    band, t, b = _band(buf, s, hy, n - hy, hy, hy)
+    compute(band, t, b, out[hy:n - hy])
+    for r in reqs:
+        r.wait()
+    # boundary bands: the top hy rows read the received top halo, and so on
+    band, t, b = _band(buf, s, 0, hy, ht, min(hy, n - hy))
+    compute(band, t, b, out[0:hy])
+    band, t, b = _band(buf, s, n - hy, n, min(hy, n - hy), hb)
+    compute(band, t, b, out[n - hy:n])
+    return out
+
+
+def _allreduce_np(a: np.ndarray, device, group=None) -> np.ndarray:
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).to(device)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t.cpu().numpy()
+
+
+def tune_pooled(frames_local, f, toq: float, metric="mre", group=None, partials=None):
+    """The TOQ tuner over the union of every rank's training frames: per-rank
+    candidate partials (paraprox_tune_partials), one all-reduce of 3 fp64 per
+    candidate, then the host-only decision (paraprox_tune_decide).  Every rank
+    holds the same sums and takes the same decision."""
+    from . import paraprox as P
+    if partials is None:
+        partials = P.tune_partials(frames_local, f, metric)
+    dev = frames_local.device if isinstance(frames_local, torch.Tensor) else "cpu"
+    summed = _allreduce_np(partials, dev if dist.get_backend(group) == "nccl" else "cpu", group)
+    return P.tune_decide(f, summed, toq, metric)
+
+
+def quality_pooled(exact, approx, metric="mre", group=None, partials=None) -> float:
+    from . import paraprox as P
+    if partials is None:
+        partials = P.quality_partials(exact, approx, metric)
+    dev = exact.device if dist.get_backend(group) == "nccl" else "cpu"
+    summed = _allreduce_np(partials, dev, group)
+    return P.quality_from_partials(summed, metric)
