@@ -153,6 +153,15 @@ PARAPROX_API paraprox_status paraprox_quality_partials(const float* d_exact, con
                                           const paraprox_image* img, paraprox_metric m,
                                           double* h_partials3, paraprox_stream s);
 
+/* Asynchronous variant: the 3 partials are written to caller-owned device
+ * memory d_partials3 (3 doubles) in stream order; nothing is copied to the
+ * host and the stream is not synchronised (runtime quality checks inside a
+ * pipeline or a CUDA graph).  Same partials, bit for bit, as
+ * paraprox_quality_partials. */
+PARAPROX_API paraprox_status paraprox_quality_partials_async(const float* d_exact, const float* d_approx,
+                                                const paraprox_image* img, paraprox_metric m,
+                                                double* d_partials3, paraprox_stream s);
+
 /* Quality from (summed) partials.  Host-only. */
 PARAPROX_API paraprox_status paraprox_quality_from_partials(const double* h_partials3, paraprox_metric m,
                                                double* h_quality);

@@ -317,6 +317,22 @@ paraprox_status paraprox_quality_partials(const float* d_exact, const float* d_a
     return quality_partials_impl(d_exact, d_approx, img, m, h_partials3, s);
 }
 
+paraprox_status paraprox_quality_partials_async(const float* d_exact, const float* d_approx,
+                                                const paraprox_image* img, paraprox_metric m, double* d_partials3,
+                                                paraprox_stream s) {
+    if (!d_exact || !d_approx || !d_partials3) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    cudaStream_t cs = (cudaStream_t)s;
+    DevBuf buf;
+    buf.s = cs;
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * 2 * kQualityBlocks, cs));
+    cudaError_t err = launch_quality(d_exact, d_approx, view_of(img), m, d_partials3, (double*)buf.p, cs);
+    if (err != cudaSuccess) return cuda_fail(err, "quality launch");
+    return PARAPROX_OK;
+}
+
 paraprox_status paraprox_quality_from_partials(const double* h_partials3, paraprox_metric m, double* h_quality) {
     if (!h_partials3 || !h_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
     if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");

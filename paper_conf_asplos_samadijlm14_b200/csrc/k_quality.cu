@@ -46,6 +46,49 @@ __device__ __forceinline__ void block_sum2(double& s0, double& s1) {
     }
 }
 
+// Contiguous images (pitch == w, frames back to back) are one flat array:
+// each thread keeps kQU independent 128-bit loads of E and of A in flight per
+// iteration (grid-stride, fixed grid), so the HBM pipe stays full while the
+// fp64 division chain of MRE runs.  Other layouts walk rows.
+constexpr int kQU = 4;
+
+template <int M>
+__global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
+                                                      long long count, double* __restrict__ part) {
+    double s0 = 0.0, s1 = 0.0;
+    const long long n4 = count >> 2;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const float4* e4 = reinterpret_cast<const float4*>(E);
+    const float4* a4 = reinterpret_cast<const float4*>(A);
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kQU * stride) {
+        float4 e[kQU], a[kQU];
+#pragma unroll
+        for (int u = 0; u < kQU; ++u) {
+            const long long j = i + u * stride;
+            if (j < n4) {
+                e[u] = __ldcs(e4 + j);
+                a[u] = __ldcs(a4 + j);
+            } else {
+                e[u] = a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kQU; ++u) {
+            accum<M>(e[u].x, a[u].x, s0, s1);
+            accum<M>(e[u].y, a[u].y, s0, s1);
+            accum<M>(e[u].z, a[u].z, s0, s1);
+            accum<M>(e[u].w, a[u].w, s0, s1);
+        }
+    }
+    if (blockIdx.x == 0)
+        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) accum<M>(E[x], A[x], s0, s1);
+    block_sum2(s0, s1);
+    if (threadIdx.x == 0) {
+        part[2 * blockIdx.x] = s0;
+        part[2 * blockIdx.x + 1] = s1;
+    }
+}
+
 template <int M>
 __global__ void __launch_bounds__(256) k_quality_partials(const float* __restrict__ E,
                                                           const float* __restrict__ A, View v,
@@ -60,12 +103,25 @@ __global__ void __launch_bounds__(256) k_quality_partials(const float* __restric
         const long long off = f * v.fstride + y * v.pitch;
         const float4* e4 = reinterpret_cast<const float4*>(E + off);
         const float4* a4 = reinterpret_cast<const float4*>(A + off);
-        for (int x = threadIdx.x; x < w4; x += blockDim.x) {
-            const float4 e = __ldcs(e4 + x), a = __ldcs(a4 + x);
-            accum<M>(e.x, a.x, s0, s1);
-            accum<M>(e.y, a.y, s0, s1);
-            accum<M>(e.z, a.z, s0, s1);
-            accum<M>(e.w, a.w, s0, s1);
+        for (int x = threadIdx.x; x < w4; x += kQU * blockDim.x) {
+            float4 e[kQU], a[kQU];
+#pragma unroll
+            for (int u = 0; u < kQU; ++u) {
+                const int j = x + u * blockDim.x;
+                if (j < w4) {
+                    e[u] = __ldcs(e4 + j);
+                    a[u] = __ldcs(a4 + j);
+                } else {
+                    e[u] = a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kQU; ++u) {
+                accum<M>(e[u].x, a[u].x, s0, s1);
+                accum<M>(e[u].y, a[u].y, s0, s1);
+                accum<M>(e[u].z, a[u].z, s0, s1);
+                accum<M>(e[u].w, a[u].w, s0, s1);
+            }
         }
         for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x)
             accum<M>(__ldcs(E + off + x), __ldcs(A + off + x), s0, s1);
@@ -103,23 +159,28 @@ __global__ void __launch_bounds__(1024) k_quality_final(const double* __restrict
 cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
                            double* d_part3, double* d_scratch, cudaStream_t s) {
     const long long rows = (long long)v.n * v.h;
-    const int g = (int)(rows < kQualityBlocks ? rows : kQualityBlocks);
     const double count = (double)v.n * (double)v.h * (double)v.w;
-    switch (m) {
-    case PARAPROX_MRE:
-        k_quality_partials<PARAPROX_MRE><<<g, 256, 0, s>>>(e, a, v, d_scratch);
-        k_quality_final<PARAPROX_MRE><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3);
-        break;
-    case PARAPROX_L2:
-        k_quality_partials<PARAPROX_L2><<<g, 256, 0, s>>>(e, a, v, d_scratch);
-        k_quality_final<PARAPROX_L2><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3);
-        break;
-    default:
-        k_quality_partials<PARAPROX_PSNR><<<g, 256, 0, s>>>(e, a, v, d_scratch);
-        k_quality_final<PARAPROX_PSNR><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3);
-        break;
+    const bool flat = v.pitch == v.w && (v.n == 1 || v.fstride == (long long)v.h * v.w) &&
+                      ((((uintptr_t)e) | ((uintptr_t)a)) & 15) == 0;
+    const long long cnt = (long long)v.n * v.h * v.w;
+    int g;
+    if (flat) {
+        const long long chunks = (cnt / 4 + 255) / 256;
+        g = (int)(chunks < kQualityBlocks ? (chunks > 0 ? chunks : 1) : kQualityBlocks);
+    } else {
+        g = (int)(rows < kQualityBlocks ? rows : kQualityBlocks);
     }
-    count_launch("quality_partials");
+#define PPX_QUALITY_CASE(M)                                                                    \
+    if (flat) k_quality_flat<M><<<g, 256, 0, s>>>(e, a, cnt, d_scratch);                       \
+    else k_quality_partials<M><<<g, 256, 0, s>>>(e, a, v, d_scratch);                          \
+    k_quality_final<M><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3);
+    switch (m) {
+    case PARAPROX_MRE: PPX_QUALITY_CASE(PARAPROX_MRE) break;
+    case PARAPROX_L2: PPX_QUALITY_CASE(PARAPROX_L2) break;
+    default: PPX_QUALITY_CASE(PARAPROX_PSNR) break;
+    }
+#undef PPX_QUALITY_CASE
+    count_launch(flat ? "quality_flat" : "quality_partials");
     count_launch("quality_final");
     return cudaGetLastError();
 }

@@ -53,6 +53,7 @@ _SIGS = {
     "paraprox_run_host": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_quality": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials": [_P, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_quality_partials_async": [_P, _P, _IMG, C.c_int, _P, _P],
     "paraprox_quality_from_partials": [_D, C.c_int, _D],
     "paraprox_tune": [_P, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
     "paraprox_tune_candidates": [_P, C.c_int, _I, _I, _I],
@@ -320,6 +321,22 @@ def quality_partials(exact, approx, metric="mre", *, stream=None) -> np.ndarray:
     _check(_lib.paraprox_quality_partials(_dp(exact), _dp(approx), C.byref(img), _metric(metric),
                                           p.ctypes.data_as(_D), _stream(stream)), "quality_partials")
     return p
+
+
+def quality_partials_async(exact, approx, metric="mre", out=None, *, stream=None) -> torch.Tensor:
+    """The 3 fp64 partials into a device tensor, stream-ordered, no sync."""
+    _need_cuda(exact, approx)
+    img = image_of(exact)
+    if exact.shape != approx.shape or exact.stride() != approx.stride():
+        raise ValueError("exact and approx must share shape and strides")
+    if out is None:
+        out = torch.empty(3, dtype=torch.float64, device=exact.device)
+    if out.dtype != torch.float64 or out.numel() < 3 or not out.is_contiguous():
+        raise ValueError("out must be a contiguous float64 device tensor of >= 3 elements")
+    _need_cuda(out)
+    _check(_lib.paraprox_quality_partials_async(_dp(exact), _dp(approx), C.byref(img), _metric(metric),
+                                                C.c_void_p(out.data_ptr()), _stream(stream)), "quality_partials_async")
+    return out
 
 
 def quality_from_partials(p, metric="mre") -> float:
