@@ -79,6 +79,25 @@ int oracle_tune(const float* x, int n, int h, int w, int separable,
                 double toq, int metric, int cap, double* qualities,
                 int* n_evaluated, int* scheme, int* reach, double* quality);
 
+/* Global-lattice reading of the stencil approximation (DESIGN.md reading
+ * G): "Paraprox accesses a subset of values in the
+ * input array and replicates that subset to construct an approximate version
+ * of the array".  Per axis of length len and reach d:
+ * the accessed coordinates are the multiples of s = 2d+1; every coordinate
+ * reads the nearest accessed one, and coordinates past the last accessed
+ * one read the last:  g[t] = min(s*floor(t/s + 1/2), s*floor((len-1)/s)).
+ * d = 0 is the identity.  Returns 0, or -1 on bad arguments. */
+int oracle_lattice_map(int len, int d, int* g);
+
+/* The approximate array X~(y,x) = X(g_y(y), g_x(x)) (reaches dy, dx), then
+ * the exact stencil (dense, or the separable two passes) applied to X~. */
+int oracle_stencil_lattice(const float* x, int n, int h, int w,
+                           const float* wgt, int ky, int kx,
+                           int dy, int dx, double* out);
+int oracle_stencil_lattice_sep(const float* x, int n, int h, int w,
+                               const float* wy, int ky, const float* wx, int kx,
+                               int dy, int dx, double* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -53,10 +53,16 @@ def lib():
         _lib.oracle_stencil_sep.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
                                             C.c_int, C.c_int, f64]
         _lib.oracle_quality.argtypes = [f64, f64, C.c_longlong, C.c_int, f64]
+        _lib.oracle_lattice_map.argtypes = [C.c_int, C.c_int, i32]
+        _lib.oracle_stencil_lattice.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, C.c_int,
+                                                C.c_int, C.c_int, f64]
+        _lib.oracle_stencil_lattice_sep.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                                    C.c_int, C.c_int, f64]
         _lib.oracle_tune_candidates.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, i32, i32]
         _lib.oracle_tune.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
                                      C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
-        for name in ("oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
+        for name in ("oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
+                     "oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
                      "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
                      "oracle_tune_candidates", "oracle_tune"):
             getattr(_lib, name).restype = C.c_int
@@ -135,6 +141,36 @@ def stencil_sep(x, wy, wx, dy: int = 0, dx: int = 0) -> np.ndarray:
     _ok(lib().oracle_stencil_sep(_fp(x), n, h, ww, _fp(wy), wy.size, _fp(wx), wx.size, dy, dx, _dp(out)),
         "stencil_sep")
     return out[0] if squeeze else out
+
+
+def lattice_map(length: int, d: int) -> np.ndarray:
+    """Global-lattice map of one axis (reading G): g[t] for t in [0, length)."""
+    g = np.zeros(max(length, 1), dtype=np.int32)
+    _ok(lib().oracle_lattice_map(int(length), int(d), g.ctypes.data_as(C.POINTER(C.c_int))), "lattice_map")
+    return g[:length]
+
+
+def stencil_lattice_xy(x, w, dy: int, dx: int) -> np.ndarray:
+    """Exact stencil on the replicated array X~ (reading G).
+    ``w`` is a 2-D array (dense) or a (wy, wx) pair (separable)."""
+    x, squeeze = _frames(x)
+    out = np.empty(x.shape, dtype=np.float64)
+    n, h, ww = x.shape
+    if isinstance(w, (tuple, list)):
+        wy = np.ascontiguousarray(w[0], dtype=np.float32).ravel()
+        wx = np.ascontiguousarray(w[1], dtype=np.float32).ravel()
+        _ok(lib().oracle_stencil_lattice_sep(_fp(x), n, h, ww, _fp(wy), wy.size, _fp(wx), wx.size, dy, dx,
+                                             _dp(out)), "stencil_lattice_sep")
+    else:
+        w = np.ascontiguousarray(w, dtype=np.float32)
+        _ok(lib().oracle_stencil_lattice(_fp(x), n, h, ww, _fp(w), w.shape[0], w.shape[1], dy, dx, _dp(out)),
+            "stencil_lattice")
+    return out[0] if squeeze else out
+
+
+def stencil_lattice(x, w, scheme, reach: int) -> np.ndarray:
+    dy, dx = scheme_reaches(scheme, reach)
+    return stencil_lattice_xy(x, w, dy, dx)
 
 
 def stencil_sep_scheme(x, wy, wx, scheme, reach: int) -> np.ndarray:
