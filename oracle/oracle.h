@@ -98,6 +98,14 @@ int oracle_stencil_lattice_sep(const float* x, int n, int h, int w,
                                const float* wy, int ky, const float* wx, int kx,
                                int dy, int dx, double* out);
 
+/* Lattice tuner: exact once, then the row lattice with reach 4, 3, 2, 1
+ * (fewest HBM bytes first); the first with quality >= toq, else EXACT.  The
+ * four qualities go to qualities4 when non-NULL. */
+int oracle_tune_lattice(const float* x, int n, int h, int w, int separable,
+                        const float* wgt_or_wy, int ky, const float* wx, int kx,
+                        double toq, int metric, double* qualities4,
+                        int* scheme, int* reach, double* quality);
+
 #ifdef __cplusplus
 }
 #endif

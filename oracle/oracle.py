@@ -61,7 +61,9 @@ def lib():
         _lib.oracle_tune_candidates.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, i32, i32]
         _lib.oracle_tune.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
                                      C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
-        for name in ("oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
+        _lib.oracle_tune_lattice.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                             C.c_double, C.c_int, f64, i32, i32, f64]
+        for name in ("oracle_tune_lattice", "oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
                      "oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
                      "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
                      "oracle_tune_candidates", "oracle_tune"):
@@ -224,3 +226,23 @@ def tune(x, w, toq: float, metric="mre", all_qualities: bool = False):
                           C.byref(q)), "tune")
     return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value,
                 qualities=[float(v) for v in qs[:nev.value]] if all_qualities else None)
+
+
+def tune_lattice(x, w, toq: float, metric="mre"):
+    """Oracle lattice tuner: row lattice reach 4, 3, 2, 1, first with quality
+    >= toq, else exact.  Returns dict(scheme, reach, quality, qualities)."""
+    x, _ = _frames(x)
+    m = METRICS[metric] if isinstance(metric, str) else int(metric)
+    n, h, ww = x.shape
+    if isinstance(w, (tuple, list)):
+        wa = np.ascontiguousarray(w[0], dtype=np.float32).ravel()
+        wb = np.ascontiguousarray(w[1], dtype=np.float32).ravel()
+        sep, ky, kx = 1, wa.size, wb.size
+    else:
+        wa = np.ascontiguousarray(w, dtype=np.float32)
+        sep, ky, kx, wb = 0, wa.shape[0], wa.shape[1], wa
+    qs = np.full(4, np.nan)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _ok(lib().oracle_tune_lattice(_fp(x), n, h, ww, sep, _fp(wa), ky, _fp(wb), kx, float(toq), m, _dp(qs),
+                                  C.byref(sc), C.byref(rc), C.byref(q)), "tune_lattice")
+    return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value, qualities=[float(v) for v in qs])

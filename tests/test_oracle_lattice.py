@@ -130,3 +130,40 @@ def test_separable_equals_dense_outer(O, dy, dx):
     np.testing.assert_allclose(O.stencil_lattice_xy(x, (wy, wx), dy, dx),
                                corr(x[0][np.ix_(O.lattice_map(33, dy), O.lattice_map(45, dx))], dense)[None],
                                rtol=1e-12, atol=1e-9)
+
+
+# ---- lattice tuner pins ---------------------------------------------------
+
+def test_tuner_constant_image_takes_sparsest(O):
+    x = np.full((2, 40, 40), 99.0, dtype=np.float32)
+    r = O.tune_lattice(x, F.mean(5), 1 - 1e-6, "mre")
+    assert (r["scheme"], r["reach"]) == ("row", 4)
+
+
+def test_tuner_y_constant_image_takes_sparsest(O):
+    row = images.random_integers((1, 64), 3).astype(np.float32)
+    x = np.repeat(row, 50, axis=0)[None]
+    r = O.tune_lattice(x, F.conv(5, seed=2), 1 - 1e-9, "l2")
+    assert (r["scheme"], r["reach"]) == ("row", 4)
+    assert all(abs(q - 1.0) < 1e-6 for q in r["qualities"])
+
+
+def test_tuner_noise_falls_back_to_exact(O):
+    x = W.uniform_noise(96, 96, 5)[None]
+    r = O.tune_lattice(x, F.mean(5), 0.95, "mre")
+    assert (r["scheme"], r["reach"], r["quality"]) == ("exact", 0, 1.0)
+
+
+def test_tuner_first_passing_and_monotone(O):
+    x = W.frames(2, 96, 128, 0)
+    w = F.gaussian(3)
+    qs = O.tune_lattice(x, w, 2.0, "mre")["qualities"]  # nothing passes: all four qualities
+    assert qs[0] <= qs[1] <= qs[2] <= qs[3] < 1.0  # sparser rows, lower quality (on these images)
+    for toq in (0.8, 0.9, 0.95, 0.99):
+        r = O.tune_lattice(x, w, toq, "mre")
+        passing = [k for k, q in enumerate(qs) if q >= toq]
+        if passing:
+            assert (r["scheme"], r["reach"]) == ("row", 4 - passing[0])
+            assert r["quality"] == qs[passing[0]]
+        else:
+            assert r["scheme"] == "exact"
