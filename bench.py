@@ -229,6 +229,7 @@ def main():
     ap.add_argument("--toq", type=float, default=0.90)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--no-lattice", action="store_true")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -282,7 +283,7 @@ def main():
     else:
         scheme, reach, q_train = P.tune(train, f, args.toq, wl["metric"])
     tune_ms = 1e3 * (time.perf_counter() - t0)
-    del train
+    train_keep = train
     plan = f.plan_info(*{"exact": (0, 0), "row": (reach, 0), "col": (0, reach),
                          "center": (reach, reach)}[scheme])
 
@@ -332,6 +333,38 @@ def main():
         exact_kernel = P.last_kernel()
         copy_ms, _, _ = timed(copy_step, args.steps, args.warmup)
 
+        # a4: the quality reduction alone (exact vs approx buffers, 8 B/px read)
+        qpart = torch.empty(3, dtype=torch.float64, device=dev)
+
+        def quality_step(k):
+            P.quality_partials_async(outputs[k % nbuf], inputs[k % nbuf], wl["metric"], qpart, stream=stream)
+
+        qual_ms, qual_kern_ms, _ = timed(quality_step, args.steps, args.warmup)
+
+        # NEXT-1: the global-lattice reading (only every (2d+1)-th row is read
+        # from HBM), tuned by its own tuner at the same TOQ on the same frames
+        lat = None
+        if not args.no_lattice:
+            if ws > 1:
+                lp = torch.from_numpy(P.tune_lattice_partials(train_keep, f, wl["metric"])).to(dev)
+                dist.all_reduce(lp)
+                l_scheme, l_reach, l_q = P.tune_lattice_decide(lp.cpu().numpy(), args.toq, wl["metric"])
+            else:
+                l_scheme, l_reach, l_q = P.tune_lattice(train_keep, f, args.toq, wl["metric"])
+            lat = {"scheme": l_scheme, "reach": l_reach, "quality_train": l_q}
+            if l_scheme != "exact":
+                lat_ops = [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=stream, lattice=True)
+                           for k in range(nbuf)]
+                lat_total, lat_kern, _ = timed(lambda k: lat_ops[k % nbuf](), args.steps, args.warmup)
+                lat_bpp = 4.0 / (2 * l_reach + 1) + 4.0
+                lat.update({
+                    "kernel": P.last_kernel(), "ms_per_step": lat_total / args.steps,
+                    "value": px_step * ws / (lat_total / args.steps * 1e-3) / 1e6, "unit": "Mpixel/s",
+                    "algorithmic_bytes_per_px": lat_bpp,
+                    "achieved_gbs": lat_bpp * px_step / (lat_kern * 1e-3) / 1e9,
+                    "speedup_vs_exact": exact_total_ms / lat_total,
+                    "speedup_vs_approx": total_ms / lat_total})
+
     ms_step = total_ms / args.steps
     value = px_step * ws / (ms_step * 1e-3) / 1e6
     exact_ms_step = exact_total_ms / args.steps
@@ -342,6 +375,14 @@ def main():
     exact_achieved = alg_bytes / (exact_kern_ms * 1e-3) / 1e9
 
     # ---- quality of the chosen configuration on the held-out frames ---------
+    if lat is not None:
+        lat["roofline_frac"] = lat.get("achieved_gbs", 0.0) / peak if "achieved_gbs" in lat else None
+        if lat["scheme"] != "exact":
+            e = P.stencil_exact(inputs[0], f)
+            a = P.stencil_lattice(inputs[0], f, lat["scheme"], lat["reach"])
+            lat["quality_heldout"] = P.quality(e, a, wl["metric"])
+            del e, a
+    del train_keep
     q_held = None
     if scheme != "exact":
         e = P.stencil_exact(inputs[0], f)
@@ -414,6 +455,11 @@ def main():
                       "kernel_gbs": exact_achieved, "roofline_frac": exact_achieved / peak, "kernel": exact_kernel},
             "copy_same_bytes_gbs": alg_bytes * args.steps / (copy_ms * 1e-3) / 1e9,
             "speedup_vs_exact": exact_ms_step / ms_step,
+            "quality_kernel": {"metric": wl["metric"], "ms": qual_kern_ms, "kernel": "quality_flat",
+                               "achieved_gbs": alg_bytes / (qual_kern_ms * 1e-3) / 1e9,
+                               "frac": alg_bytes / (qual_kern_ms * 1e-3) / 1e9 / peak,
+                               "note": "a4 alone: reads E and A (8 B/px), fp64 partials, 2 launches"},
+            "lattice": lat,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": load_traffic(args.workload, approx_kernel),
                          "kernel": approx_kernel, "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",

@@ -128,6 +128,24 @@ PARAPROX_API paraprox_status paraprox_stencil_approx_xy(paraprox_filter f, int r
                                            const float* d_in, float* d_out,
                                            const paraprox_image* img, paraprox_stream s);
 
+/* Global-lattice reading (reading G):
+ * "Paraprox accesses a subset of values in the input array and replicates
+ * that subset to construct an approximate version of the array" (PAPER.md
+ * L350-356).  Per axis with reach d >= 1 the accessed coordinates are the
+ * multiples of s = 2d+1; every coordinate reads the nearest accessed one
+ * (those past the last accessed one read the last), and the exact stencil is
+ * applied to that array.  Schemes: row = (d, 0), column = (0, d), centre =
+ * (d, d); reach 0 or EXACT = the exact stencil.  The row lattice reads only
+ * every s-th row from HBM (4/s + 4 bytes per output pixel).  halo_top and
+ * halo_bottom must be 0 (the lattice is anchored at row 0 of each frame).
+ * Reaches above 2^20 are INVALID_ARG.  Asynchronous on s. */
+PARAPROX_API paraprox_status paraprox_stencil_lattice(paraprox_filter f, paraprox_scheme scheme, int reach,
+                                         const float* d_in, float* d_out,
+                                         const paraprox_image* img, paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_stencil_lattice_xy(paraprox_filter f, int reach_y, int reach_x,
+                                            const float* d_in, float* d_out,
+                                            const paraprox_image* img, paraprox_stream s);
+
 /* End-to-end convenience over HOST buffers: copies h_in to the device,
  * runs the stencil (scheme, reach), copies the result to h_out, overlapping
  * the transfers with the kernels chunk by chunk.  Pinned host memory gives
@@ -193,6 +211,22 @@ PARAPROX_API paraprox_status paraprox_tune_partials(paraprox_filter f, const flo
 PARAPROX_API paraprox_status paraprox_tune_decide(paraprox_filter f, const double* h_partials,
                                      paraprox_metric m, double toq, paraprox_scheme* out_scheme,
                                      int* out_reach, double* out_quality);
+
+/* Lattice tuner: the exact stencil once on d_train, then the row lattice
+ * with reach 4, 3, 2, 1 (fewest HBM bytes first); the first whose quality
+ * >= toq wins, else (EXACT, 0, 1.0 / +inf dB).  Syncs s.  Its multi-GPU split:
+ * 3 partials per candidate (12 doubles, candidate order) for the local
+ * frames, then a host-only decision from the (all-reduced) partials. */
+PARAPROX_API paraprox_status paraprox_tune_lattice(paraprox_filter f, const float* d_train,
+                                      const paraprox_image* img, double toq, paraprox_metric m,
+                                      paraprox_scheme* out_scheme, int* out_reach, double* out_quality,
+                                      paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_tune_lattice_partials(paraprox_filter f, const float* d_train,
+                                               const paraprox_image* img, paraprox_metric m,
+                                               double* h_partials12, paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_tune_lattice_decide(const double* h_partials12, paraprox_metric m,
+                                             double toq, paraprox_scheme* out_scheme, int* out_reach,
+                                             double* out_quality);
 
 /* ---- diagnostics -------------------------------------------------------- */
 

@@ -93,6 +93,26 @@ static paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const floa
     return PARAPROX_OK;
 }
 
+constexpr int kMaxLatticeReach = 1 << 20;
+
+static paraprox_status run_lattice(paraprox_filter f, int dy, int dx, const float* in, float* out,
+                                   const paraprox_image* img, paraprox_stream s) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    if (!in || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL buffer");
+    if (dy < 0 || dx < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    if (dy > kMaxLatticeReach || dx > kMaxLatticeReach) return fail(PARAPROX_ERR_INVALID_ARG, "reach too large");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    if (overlaps(in, out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_in");
+    const View v = view_of(img);
+    const long long ofs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
+    cudaError_t e = (dy == 0 && dx == 0)
+                        ? launch_stencil(get_plan(f, 0, 0), in, v, out, img->pitch, ofs, (cudaStream_t)s)
+                        : launch_lattice(*f, in, v, out, img->pitch, ofs, dy, dx, (cudaStream_t)s);
+    if (e != cudaSuccess) return cuda_fail(e, "lattice launch");
+    return PARAPROX_OK;
+}
+
 static double quality_of(const double* p3, paraprox_metric m) {
     if (m == PARAPROX_MRE) return 1.0 - p3[0] / p3[1];
     if (m == PARAPROX_L2) {
@@ -200,6 +220,49 @@ static paraprox_status tune_partials_impl(paraprox_filter f, const float* d_trai
     return PARAPROX_OK;
 }
 
+// the lattice tuner's candidates: row lattice reach 4, 3, 2, 1 (fewest HBM
+// bytes first, 4/(2d+1) + 4 B per pixel)
+constexpr int kLatticeCands = 4;
+
+static paraprox_status lattice_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                                             paraprox_metric m, double* h_partials, paraprox_stream s) {
+    if (!f || !d_train || !h_partials) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    cudaStream_t cs = (cudaStream_t)s;
+    const long long plane = (long long)img->h * img->w;
+    const long long count = plane * img->n;
+    DevBuf buf;
+    buf.s = cs;
+    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (2 * kQualityBlocks + 3 * kLatticeCands) + 256;
+    PPX_CUDA(scratch_alloc(&buf.p, bytes, cs));
+    float* E = (float*)buf.p;
+    float* A = E + count;
+    double* scratch = (double*)(((uintptr_t)(A + count) + 255) & ~(uintptr_t)255);
+    double* parts = scratch + 2 * kQualityBlocks;
+    const View vin = view_of(img);
+    View vq;
+    vq.n = img->n;
+    vq.h = img->h;
+    vq.w = img->w;
+    vq.pitch = img->w;
+    vq.fstride = plane;
+    vq.lo = 0;
+    vq.hi = img->h - 1;
+    cudaError_t e = launch_stencil(get_plan(f, 0, 0), d_train, vin, E, img->w, plane, cs);
+    if (e != cudaSuccess) return cuda_fail(e, "exact launch");
+    for (int k = 0; k < kLatticeCands; ++k) {
+        e = launch_lattice(*f, d_train, vin, A, img->w, plane, kLatticeCands - k, 0, cs);
+        if (e != cudaSuccess) return cuda_fail(e, "lattice launch");
+        e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);
+        if (e != cudaSuccess) return cuda_fail(e, "quality launch");
+    }
+    PPX_CUDA(cudaMemcpyAsync(h_partials, parts, sizeof(double) * 3 * kLatticeCands, cudaMemcpyDeviceToHost, cs));
+    PPX_CUDA(cudaStreamSynchronize(cs));
+    return PARAPROX_OK;
+}
+
 static paraprox_status decide(const std::vector<Candidate>& cands, const double* parts, paraprox_metric m,
                               double toq, paraprox_scheme* sc, int* reach, double* q) {
     *sc = PARAPROX_EXACT;
@@ -300,6 +363,57 @@ paraprox_status paraprox_stencil_approx(paraprox_filter f, paraprox_scheme schem
 paraprox_status paraprox_stencil_approx_xy(paraprox_filter f, int reach_y, int reach_x, const float* d_in,
                                            float* d_out, const paraprox_image* img, paraprox_stream s) {
     return run_stencil(f, reach_y, reach_x, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_stencil_lattice(paraprox_filter f, paraprox_scheme scheme, int reach, const float* d_in,
+                                         float* d_out, const paraprox_image* img, paraprox_stream s) {
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    return run_lattice(f, dy, dx, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_stencil_lattice_xy(paraprox_filter f, int reach_y, int reach_x, const float* d_in,
+                                            float* d_out, const paraprox_image* img, paraprox_stream s) {
+    return run_lattice(f, reach_y, reach_x, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_tune_lattice_partials(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                                               paraprox_metric m, double* h_partials12, paraprox_stream s) {
+    return lattice_partials_impl(f, d_train, img, m, h_partials12, s);
+}
+
+paraprox_status paraprox_tune_lattice_decide(const double* h_partials12, paraprox_metric m, double toq,
+                                             paraprox_scheme* out_scheme, int* out_reach, double* out_quality) {
+    if (!h_partials12 || !out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    *out_scheme = PARAPROX_EXACT;
+    *out_reach = 0;
+    *out_quality = m == PARAPROX_PSNR ? INFINITY : 1.0;
+    for (int k = 0; k < kLatticeCands; ++k) {
+        const double q = quality_of(h_partials12 + 3 * k, m);
+        if (q >= toq) {
+            *out_scheme = PARAPROX_ROW;
+            *out_reach = kLatticeCands - k;
+            *out_quality = q;
+            break;
+        }
+    }
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_tune_lattice(paraprox_filter f, const float* d_train, const paraprox_image* img, double toq,
+                                      paraprox_metric m, paraprox_scheme* out_scheme, int* out_reach,
+                                      double* out_quality, paraprox_stream s) {
+    if (!out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    double parts[3 * kLatticeCands];
+    st = lattice_partials_impl(f, d_train, img, m, parts, s);
+    if (st != PARAPROX_OK) return st;
+    return paraprox_tune_lattice_decide(parts, m, toq, out_scheme, out_reach, out_quality);
 }
 
 paraprox_status paraprox_quality(const float* d_exact, const float* d_approx, const paraprox_image* img,

@@ -1,5 +1,6 @@
 // dispatch.cu -- picks the kernel variant for a plan and an image layout.
 //
+// Centre-only plans (full collapse, or 1x1 filters) are maps: k_pointwise.cu.
 // Fast path: the persistent TMA tile kernel instance (k_tiles.cuh) whose
 // compile-time accessed-offset masks equal the plan's (every plan of a filter
 // up to 9x9 has one; instances are registered by inst_r*_*.cu).  It needs a
@@ -16,6 +17,8 @@ namespace ppx {
 
 cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float* out, long long opitch,
                            long long ofs, cudaStream_t s);
+cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, float* out, long long opitch,
+                             long long ofs, cudaStream_t s);
 
 void register_r1_dense();
 void register_r2_dense();
@@ -151,6 +154,8 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
 
 cudaError_t launch_stencil(const Plan& p, const float* in, const View& v, float* out, long long opitch,
                            long long ofs, cudaStream_t s) {
+    // a plan that accesses only the centre is a map: stream it (k_pointwise.cu)
+    if (!force_generic() && p.hy == 0 && p.hx == 0) return launch_pointwise(p, in, v, out, opitch, ofs, s);
     if (!force_generic() && p.ry <= 4 && p.rx <= 4) {
         init_registry();
         for (Entry& e : reg()) {

@@ -76,6 +76,10 @@ struct View {
 // name and returns cudaGetLastError().
 cudaError_t launch_stencil(const Plan& p, const float* in, const View& vin, float* out,
                            long long out_pitch, long long out_fstride, cudaStream_t s);
+// global-lattice stencil (k_lattice.cu): exact stencil on the array rebuilt
+// from the accessed rows/columns (reaches dy, dx); halos must be 0
+cudaError_t launch_lattice(const paraprox_filter_s& f, const float* in, const View& v, float* out,
+                           long long out_pitch, long long out_fstride, int dy, int dx, cudaStream_t s);
 cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
                            double* d_part3, double* d_scratch, cudaStream_t s);
 constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums

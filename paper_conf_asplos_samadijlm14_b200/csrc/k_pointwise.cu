@@ -1,0 +1,117 @@
+// k_pointwise.cu -- plans whose accessed offsets are only (0, 0).
+//
+// At full reach the centre scheme lets the tile centre stand in for every
+// neighbour ("the center element ... approximates all neighboring values",
+// PAPER.md L1158-1162 Fig. 6a): the folded filter is one tap w' = sum of all
+// weights, so the stencil degenerates to the map out = w' * in -- no halo, no
+// neighbour, nothing to stage.  This kernel streams it at copy speed: each
+// thread keeps kPU independent 128-bit loads in flight (evict-first), grid =
+// resident threads, 128-bit streaming stores.  8 B of HBM per pixel.
+//
+// Rounding matches the tile kernels bit for bit: dense fmaf(w, x, 0);
+// separable fmaf(wy, fmaf(wx, x, 0), 0) (horizontal, then vertical pass).
+#include "internal.h"
+
+namespace ppx {
+
+constexpr int kPU = 4;
+
+template <bool SEP>
+__device__ __forceinline__ float pw(float x, float w0, float w1) {
+    if constexpr (SEP) return __fmaf_rn(w0, __fmaf_rn(w1, x, 0.f), 0.f);
+    else return __fmaf_rn(w0, x, 0.f);
+}
+
+template <bool SEP>
+__device__ __forceinline__ float4 pw4(float4 x, float w0, float w1) {
+    return make_float4(pw<SEP>(x.x, w0, w1), pw<SEP>(x.y, w0, w1), pw<SEP>(x.z, w0, w1), pw<SEP>(x.w, w0, w1));
+}
+
+// contiguous input and output, 16-byte aligned: one flat array
+template <bool SEP>
+__global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict__ in, float* __restrict__ out,
+                                                        long long count, float w0, float w1) {
+    const long long n4 = count >> 2;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const float4* i4 = reinterpret_cast<const float4*>(in);
+    float4* o4 = reinterpret_cast<float4*>(out);
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kPU * stride) {
+        float4 v[kPU];
+#pragma unroll
+        for (int u = 0; u < kPU; ++u)
+            if (i + u * stride < n4) v[u] = __ldcs(i4 + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < kPU; ++u)
+            if (i + u * stride < n4) __stcs(o4 + i + u * stride, pw4<SEP>(v[u], w0, w1));
+    }
+    if (blockIdx.x == 0)
+        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) out[x] = pw<SEP>(in[x], w0, w1);
+}
+
+// any layout: rows of the output image, 128-bit where both rows allow it
+template <bool SEP>
+__global__ void __launch_bounds__(256) k_pointwise_rows(const float* __restrict__ in, View v,
+                                                        float* __restrict__ out, long long opitch,
+                                                        long long ofs, float w0, float w1) {
+    const long long rows = (long long)v.n * v.h;
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    for (long long R = blockIdx.x; R < rows; R += gridDim.x) {
+        const long long f = R / v.h, y = R - f * v.h;
+        const float* src = in + f * v.fstride + y * v.pitch;
+        float* dst = out + f * ofs + y * opitch;
+        const bool vec = ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15) == 0;
+        const int w4 = vec ? (v.w >> 2) : 0;
+        for (int x = threadIdx.x; x < w4; x += blockDim.x)
+            __stcs(reinterpret_cast<float4*>(dst) + x, pw4<SEP>(__ldcs(reinterpret_cast<const float4*>(src) + x), w0, w1));
+        for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x) __stcs(dst + x, pw<SEP>(__ldcs(src + x), w0, w1));
+    }
+}
+
+cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, float* out, long long opitch,
+                             long long ofs, cudaStream_t s) {
+    static int sms[64] = {};
+    int dev = 0;
+    cudaError_t err = cudaGetDevice(&dev);
+    if (err != cudaSuccess) return err;
+    int nsm = dev < 64 ? sms[dev] : 0;
+    if (!nsm) {
+        err = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        if (err != cudaSuccess) return err;
+        if (dev < 64) sms[dev] = nsm;
+    }
+    const float w0 = p.separable ? p.wyf[0] : p.wf[0];
+    const float w1 = p.separable ? p.wxf[0] : 1.f;
+    const long long count = (long long)v.n * v.h * v.w;
+    const bool flat = v.pitch == v.w && opitch == v.w && (v.n == 1 || (v.fstride == (long long)v.h * v.w &&
+                      ofs == (long long)v.h * v.w)) &&
+                      (((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15) == 0);
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(256);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    const long long resident = (long long)nsm * 8;  // 2048 threads per SM
+    if (flat) {
+        const long long want = (count / 4 + 255) / 256;
+        cfg.gridDim = dim3((unsigned)(want < resident ? (want > 0 ? want : 1) : resident));
+        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_flat<true>, in, out, count, w0, w1)
+                          : cudaLaunchKernelEx(&cfg, k_pointwise_flat<false>, in, out, count, w0, w1);
+        count_launch(p.separable ? "sep_map" : "dense_map");
+    } else {
+        const long long rows = (long long)v.n * v.h;
+        cfg.gridDim = dim3((unsigned)(rows < resident ? rows : resident));
+        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_rows<true>, in, v, out, opitch, ofs, w0, w1)
+                          : cudaLaunchKernelEx(&cfg, k_pointwise_rows<false>, in, v, out, opitch, ofs, w0, w1);
+        count_launch(p.separable ? "sep_map_rows" : "dense_map_rows");
+    }
+    if (err != cudaSuccess) return err;
+    return cudaGetLastError();
+}
+
+}  // namespace ppx

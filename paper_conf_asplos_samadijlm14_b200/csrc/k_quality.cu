@@ -1,7 +1,8 @@
 // k_quality.cu -- output-quality partial sums (Table 1
 // metrics): mean relative error, L2-norm, PSNR.
 //
-// fp32 inputs, fp64 accumulation.  Deterministic: a fixed number of CTAs
+// fp32 inputs; fp64 per-thread sums (MRE terms formed as fp32 pairs), fp64
+// reductions.  Deterministic: a fixed number of CTAs
 // (kQualityBlocks, or fewer rows), each walking its rows in a fixed order,
 // fixed warp-shuffle trees, then one CTA summing the per-CTA partials in a
 // fixed order.  No atomics.  8 bytes of HBM read per pixel, nothing written.
@@ -9,19 +10,79 @@
 
 namespace ppx {
 
+// Per-thread accumulators.  L2 / PSNR: fp64 (the difference of two fp32
+// values is exact in fp64; 2 DFMA per pixel).  MRE needs a quotient per
+// pixel, and fp64 division is far below the HBM rate on this part (the first
+// version ran at ~1.5 TB/s), so each term |A-E|/|E| is formed as an unevaluated
+// fp32 pair q0 + q1 (exact difference by TwoSum, quotient by the approximate
+// fp32 reciprocal plus one FMA remainder correction, relative error ~2^-46)
+// whose two parts are summed in two fp64 accumulators.  Terms the pair arithmetic cannot carry (|E| tiny, |A-E| huge) take
+// the fp64 path.  Tests bound the result against the fp64 oracle at 1e-12.
 template <int M>
-__device__ __forceinline__ void accum(float e, float a, double& s0, double& s1) {
-    const double de = (double)e, da = (double)a;
-    const double d = da - de;
-    if (M == PARAPROX_MRE) {
-        s0 += de != 0.0 ? fabs(d) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
-    } else if (M == PARAPROX_L2) {
-        s0 += d * d;
-        s1 += de * de;
-    } else {
-        s0 += d * d;
+struct QAcc {
+    double s0 = 0.0, s1 = 0.0;
+    __device__ __forceinline__ void add(float e, float a) {
+        const double de = (double)e, da = (double)a;
+        const double d = da - de;
+        if (M == PARAPROX_L2) {
+            s0 = fma(d, d, s0);
+            s1 = fma(de, de, s1);
+        } else {
+            s0 = fma(d, d, s0);
+        }
     }
+    __device__ __forceinline__ void get(double& a, double& b) const {
+        a = s0;
+        b = s1;
+    }
+};
+
+__device__ __forceinline__ void two_sum(float a, float b, float& s, float& err) {
+    s = __fadd_rn(a, b);
+    const float bb = __fsub_rn(s, a);
+    err = __fadd_rn(__fsub_rn(a, __fsub_rn(s, bb)), __fsub_rn(b, bb));
 }
+
+__device__ __forceinline__ float rcp_approx(float x) {
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+
+template <>
+struct QAcc<PARAPROX_MRE> {
+    double hi = 0.0, lo = 0.0;  // sums of the leading and trailing parts of the terms
+    __device__ __forceinline__ void add_slow(float e, float a) {
+        const double de = (double)e, da = (double)a;
+        const double q = de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
+        hi += q;
+    }
+    __device__ __forceinline__ void add(float e, float a) {
+        float dh, dl;
+        two_sum(a, -e, dh, dl);  // A - E exactly, as dh + dl
+        const float ae = fabsf(e);
+        if (ae >= 1e-30f && ae <= 1e30f && fabsf(dh) <= 1e30f) {
+            if (dh < 0.f) {
+                dh = -dh;
+                dl = -dl;
+            }
+            // q0 + q1 = |A-E| / |E| to ~2^-46: the remainder of the first
+            // quotient is exact under the FMA, so the approximate reciprocal's
+            // own error is corrected by the second term
+            const float rc = rcp_approx(ae);
+            const float q0 = __fmul_rn(dh, rc);
+            const float rem = __fadd_rn(__fmaf_rn(-q0, ae, dh), dl);
+            hi += (double)q0;
+            lo += (double)__fmul_rn(rem, rc);
+        } else {  // rare: fp64 quotient (or the E == 0 convention, S12)
+            add_slow(e, a);
+        }
+    }
+    __device__ __forceinline__ void get(double& a, double& b) const {
+        a = hi + lo;
+        b = 0.0;
+    }
+};
 
 __device__ __forceinline__ void block_sum2(double& s0, double& s1) {
     __shared__ double red[2][32];
@@ -55,7 +116,7 @@ constexpr int kQU = 4;
 template <int M>
 __global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
                                                       long long count, double* __restrict__ part) {
-    double s0 = 0.0, s1 = 0.0;
+    QAcc<M> q;
     const long long n4 = count >> 2;
     const long long stride = (long long)gridDim.x * blockDim.x;
     const float4* e4 = reinterpret_cast<const float4*>(E);
@@ -74,14 +135,16 @@ __global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ 
         }
 #pragma unroll
         for (int u = 0; u < kQU; ++u) {
-            accum<M>(e[u].x, a[u].x, s0, s1);
-            accum<M>(e[u].y, a[u].y, s0, s1);
-            accum<M>(e[u].z, a[u].z, s0, s1);
-            accum<M>(e[u].w, a[u].w, s0, s1);
+            q.add(e[u].x, a[u].x);
+            q.add(e[u].y, a[u].y);
+            q.add(e[u].z, a[u].z);
+            q.add(e[u].w, a[u].w);
         }
     }
     if (blockIdx.x == 0)
-        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) accum<M>(E[x], A[x], s0, s1);
+        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) q.add(E[x], A[x]);
+    double s0, s1;
+    q.get(s0, s1);
     block_sum2(s0, s1);
     if (threadIdx.x == 0) {
         part[2 * blockIdx.x] = s0;
@@ -93,7 +156,7 @@ template <int M>
 __global__ void __launch_bounds__(256) k_quality_partials(const float* __restrict__ E,
                                                           const float* __restrict__ A, View v,
                                                           double* __restrict__ part) {
-    double s0 = 0.0, s1 = 0.0;
+    QAcc<M> q;
     const long long rows = (long long)v.n * v.h;
     const bool vec = ((v.pitch & 3) == 0) && ((v.fstride & 3) == 0) &&
                      ((((uintptr_t)E) | ((uintptr_t)A)) & 15) == 0;
@@ -117,15 +180,17 @@ __global__ void __launch_bounds__(256) k_quality_partials(const float* __restric
             }
 #pragma unroll
             for (int u = 0; u < kQU; ++u) {
-                accum<M>(e[u].x, a[u].x, s0, s1);
-                accum<M>(e[u].y, a[u].y, s0, s1);
-                accum<M>(e[u].z, a[u].z, s0, s1);
-                accum<M>(e[u].w, a[u].w, s0, s1);
+                q.add(e[u].x, a[u].x);
+                q.add(e[u].y, a[u].y);
+                q.add(e[u].z, a[u].z);
+                q.add(e[u].w, a[u].w);
             }
         }
         for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x)
-            accum<M>(__ldcs(E + off + x), __ldcs(A + off + x), s0, s1);
+            q.add(__ldcs(E + off + x), __ldcs(A + off + x));
     }
+    double s0, s1;
+    q.get(s0, s1);
     block_sum2(s0, s1);
     if (threadIdx.x == 0) {
         part[2 * blockIdx.x] = s0;

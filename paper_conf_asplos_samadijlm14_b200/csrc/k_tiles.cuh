@@ -25,6 +25,9 @@
 //  * Outputs leave as 128-bit streaming stores (st.global.cs).
 #pragma once
 
+#include <type_traits>
+#include <utility>
+
 #include "internal.h"
 #include "tma.cuh"
 
@@ -77,17 +80,45 @@ __device__ __forceinline__ constexpr bool row_needed(int rr) {
     return false;
 }
 
+// A thread's staged row segment v[0..NV-1] (its 4 columns plus the halo) as
+// even pairs ve[m] = (v[2m], v[2m+1]) straight from 128-bit LDS, and odd pairs
+// vo[m] = (v[2m+1], v[2m+2]) for offsets that start on an odd column.
 template <int NV>
-__device__ __forceinline__ void load_row(const float* row, int lane, float (&v)[NV]) {
+__device__ __forceinline__ void load_pairs(const float* row, int lane, float2 (&ve)[NV / 2],
+                                           float2 (&vo)[NV / 2 - 1]) {
     const float4* p = reinterpret_cast<const float4*>(row) + lane;
 #pragma unroll
     for (int q = 0; q < NV / 4; ++q) {
         const float4 t = p[q];
-        v[4 * q + 0] = t.x;
-        v[4 * q + 1] = t.y;
-        v[4 * q + 2] = t.z;
-        v[4 * q + 3] = t.w;
+        ve[2 * q] = make_float2(t.x, t.y);
+        ve[2 * q + 1] = make_float2(t.z, t.w);
     }
+#pragma unroll
+    for (int m = 0; m < NV / 2 - 1; ++m) vo[m] = make_float2(ve[m].y, ve[m + 1].x);
+}
+
+// acc[0] += w * (v[I0], v[I0+1]); acc[1] += w * (v[I0+2], v[I0+3])
+template <int NV, int I0>
+__device__ __forceinline__ void fma_pairs(float2 (&acc)[2], float w, const float2 (&ve)[NV / 2],
+                                          const float2 (&vo)[NV / 2 - 1]) {
+    const float2 w2 = make_float2(w, w);
+    if constexpr ((I0 & 1) == 0) {
+        acc[0] = __ffma2_rn(w2, ve[I0 >> 1], acc[0]);
+        acc[1] = __ffma2_rn(w2, ve[(I0 >> 1) + 1], acc[1]);
+    } else {
+        acc[0] = __ffma2_rn(w2, vo[I0 >> 1], acc[0]);
+        acc[1] = __ffma2_rn(w2, vo[(I0 >> 1) + 1], acc[1]);
+    }
+}
+
+// compile-time loop: f(std::integral_constant<int, 0>) ... f(<N-1>)
+template <class F, int... Is>
+__device__ __forceinline__ void static_for_impl(F&& f, std::integer_sequence<int, Is...>) {
+    (f(std::integral_constant<int, Is>{}), ...);
+}
+template <int N, class F>
+__device__ __forceinline__ void static_for(F&& f) {
+    static_for_impl(f, std::make_integer_sequence<int, N>{});
 }
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
@@ -153,59 +184,62 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         const int clo = max(0, HXP - x0);
         const int chi = min(SW - 1, A.w - 1 - x0 + HXP);
         if (clo > 0 || chi < SW - 1) {  // border columns: replicate the edge (clamp)
-            for (int idx = tid; idx < SH * SW; idx += kThreads) {
-                const int r = idx / SW, c = idx - r * SW;
-                if (c < clo) S[r * SW + c] = S[r * SW + clo];
-                else if (c > chi) S[r * SW + c] = S[r * SW + chi];
+            // only the out-of-image columns are touched: at most HXP per side
+            const int nl = clo, nr = SW - 1 - chi, nb = nl + nr;
+            for (int idx = tid; idx < SH * nb; idx += kThreads) {
+                const int r = idx / nb, c = idx - r * nb;
+                if (c < nl) S[r * SW + c] = S[r * SW + clo];
+                else S[r * SW + chi + 1 + (c - nl)] = S[r * SW + chi];
             }
             __syncthreads();
         }
 
         const int ty0 = wi * kRB;
-        float acc[kRB][4];
+        // outputs as column pairs (c = 0,1 and 2,3): every FMA is a packed
+        // FFMA2 (fma.rn.f32x2, sm_100) -- the same fp32 fma per lane, so the
+        // per-pixel rounding and tap order are unchanged, at half the issue
+        // slots
+        float2 acc[kRB][2];
 #pragma unroll
-        for (int k = 0; k < kRB; ++k) acc[k][0] = acc[k][1] = acc[k][2] = acc[k][3] = 0.f;
+        for (int k = 0; k < kRB; ++k) acc[k][0] = acc[k][1] = make_float2(0.f, 0.f);
 
         if constexpr (!SEP) {
-#pragma unroll
-            for (int rr = 0; rr < kRB + 2 * HY; ++rr) {
-                if (!row_needed<MASKY, HY>(rr)) continue;
-                const int sr = min(max(ty0 + rr, rlo), rhi);
-                float v[NV];
-                load_row<NV>(S + sr * SW, lane, v);
-#pragma unroll
-                for (int k = 0; k < kRB; ++k) {
-                    const int a = rr - HY - k;
-                    if (a < -HY || a > HY || !has(MASKY, a)) continue;
-#pragma unroll
-                    for (int b = -HX; b <= HX; ++b) {
-                        if (!has(MASKX, b)) continue;
-                        const float wt = W.w[a + 4][b + 4];
-#pragma unroll
-                        for (int c = 0; c < 4; ++c) acc[k][c] = fmaf(wt, v[HXP + c + b], acc[k][c]);
-                    }
+            // fully unrolled at compile time (static_for): the weights are
+            // kernel-parameter constants at fixed offsets, no indexed loads
+            static_for<kRB + 2 * HY>([&](auto RR) {
+                constexpr int rr = decltype(RR)::value;
+                if constexpr (row_needed<MASKY, HY>(rr)) {
+                    const int sr = min(max(ty0 + rr, rlo), rhi);
+                    float2 ve[NV / 2], vo[NV / 2 - 1];
+                    load_pairs<NV>(S + sr * SW, lane, ve, vo);
+                    static_for<kRB>([&](auto K) {
+                        constexpr int k = decltype(K)::value;
+                        constexpr int a = rr - HY - k;
+                        if constexpr (a >= -HY && a <= HY && has(MASKY, a)) {
+                            static_for<2 * HX + 1>([&](auto B) {
+                                constexpr int b = decltype(B)::value - HX;
+                                if constexpr (has(MASKX, b)) fma_pairs<NV, HXP + b>(acc[k], W.w[a + 4][b + 4], ve, vo);
+                            });
+                        }
+                    });
                 }
-            }
+            });
         } else {
             // horizontal pass over the staged rows (clamped), kept in registers
             constexpr int RPT = (SH + kWarps - 1) / kWarps;  // rows per thread
-            float hz[RPT][4];
+            float2 hz[RPT][2];
 #pragma unroll
             for (int q = 0; q < RPT; ++q) {
                 const int r = wi + q * kWarps;
                 if (r < SH) {
                     const int sr = min(max(r, rlo), rhi);
-                    float v[NV];
-                    load_row<NV>(S + sr * SW, lane, v);
-#pragma unroll
-                    for (int c = 0; c < 4; ++c) hz[q][c] = 0.f;
-#pragma unroll
-                    for (int b = -HX; b <= HX; ++b) {
-                        if (!has(MASKX, b)) continue;
-                        const float wt = W.wx[b + 4];
-#pragma unroll
-                        for (int c = 0; c < 4; ++c) hz[q][c] = fmaf(wt, v[HXP + c + b], hz[q][c]);
-                    }
+                    float2 ve[NV / 2], vo[NV / 2 - 1];
+                    load_pairs<NV>(S + sr * SW, lane, ve, vo);
+                    hz[q][0] = hz[q][1] = make_float2(0.f, 0.f);
+                    static_for<2 * HX + 1>([&](auto B) {
+                        constexpr int b = decltype(B)::value - HX;
+                        if constexpr (has(MASKX, b)) fma_pairs<NV, HXP + b>(hz[q], W.wx[b + 4], ve, vo);
+                    });
                 }
             }
             __syncthreads();  // every thread has read its rows: overwrite in place
@@ -213,7 +247,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
             for (int q = 0; q < RPT; ++q) {
                 const int r = wi + q * kWarps;
                 if (r < SH)
-                    reinterpret_cast<float4*>(S + r * SW + HXP)[lane] = make_float4(hz[q][0], hz[q][1], hz[q][2], hz[q][3]);
+                    reinterpret_cast<float4*>(S + r * SW + HXP)[lane] =
+                        make_float4(hz[q][0].x, hz[q][0].y, hz[q][1].x, hz[q][1].y);
             }
             __syncthreads();
             // vertical pass (rows already clamped by the horizontal pass)
@@ -221,15 +256,15 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
             for (int rr = 0; rr < kRB + 2 * HY; ++rr) {
                 if (!row_needed<MASKY, HY>(rr)) continue;
                 const float4 t = reinterpret_cast<const float4*>(S + (ty0 + rr) * SW + HXP)[lane];
+                const float2 t0 = make_float2(t.x, t.y), t1 = make_float2(t.z, t.w);
 #pragma unroll
                 for (int k = 0; k < kRB; ++k) {
                     const int a = rr - HY - k;
                     if (a < -HY || a > HY || !has(MASKY, a)) continue;
                     const float wt = W.wy[a + 4];
-                    acc[k][0] = fmaf(wt, t.x, acc[k][0]);
-                    acc[k][1] = fmaf(wt, t.y, acc[k][1]);
-                    acc[k][2] = fmaf(wt, t.z, acc[k][2]);
-                    acc[k][3] = fmaf(wt, t.w, acc[k][3]);
+                    const float2 w2 = make_float2(wt, wt);
+                    acc[k][0] = __ffma2_rn(w2, t0, acc[k][0]);
+                    acc[k][1] = __ffma2_rn(w2, t1, acc[k][1]);
                 }
             }
         }
@@ -243,11 +278,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
             if (y < A.h && x < A.w) {
                 float* o = obase + (long long)y * A.opitch;
                 if (x + 3 < A.w) {
-                    __stcs(reinterpret_cast<float4*>(o), make_float4(acc[k][0], acc[k][1], acc[k][2], acc[k][3]));
+                    __stcs(reinterpret_cast<float4*>(o), make_float4(acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y));
                 } else {
+                    const float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
 #pragma unroll
                     for (int c = 0; c < 4; ++c)
-                        if (x + c < A.w) __stcs(o + c, acc[k][c]);
+                        if (x + c < A.w) __stcs(o + c, r4[c]);
                 }
             }
         }

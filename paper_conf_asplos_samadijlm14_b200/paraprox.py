@@ -16,7 +16,7 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libparaprox.so")
+LIB_PATH = os.environ.get("PARAPROX_LIB") or os.path.join(_HERE, "libparaprox.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`")
@@ -51,6 +51,11 @@ _SIGS = {
     "paraprox_stencil_approx": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_stencil_approx_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_run_host": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_stencil_lattice": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_stencil_lattice_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_tune_lattice": [_P, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
+    "paraprox_tune_lattice_partials": [_P, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_tune_lattice_decide": [_D, C.c_int, C.c_double, _I, _I, _D],
     "paraprox_quality": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials_async": [_P, _P, _IMG, C.c_int, _P, _P],
@@ -263,19 +268,44 @@ def stencil_approx_xy(x, f: Filter, reach_y: int, reach_x: int, out=None, *, hal
     return out
 
 
+def stencil_lattice(x, f: Filter, scheme, reach: int, out=None, *, stream=None):
+    """Global-lattice reading: the exact stencil on the
+    array rebuilt from every (2*reach+1)-th row / column / both."""
+    _need_cuda(x)
+    img = image_of(x)
+    out = _out_like(x, 0, 0, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_lattice(f.handle, _scheme(scheme), int(reach), _dp(x), _dp(out), C.byref(img),
+                                         _stream(stream)), "stencil_lattice")
+    return out
+
+
+def stencil_lattice_xy(x, f: Filter, reach_y: int, reach_x: int, out=None, *, stream=None):
+    _need_cuda(x)
+    img = image_of(x)
+    out = _out_like(x, 0, 0, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_lattice_xy(f.handle, int(reach_y), int(reach_x), _dp(x), _dp(out), C.byref(img),
+                                            _stream(stream)), "stencil_lattice_xy")
+    return out
+
+
 class Prepared:
     """A stencil call with its arguments marshalled once (for tight loops and
     graph capture): calling it re-issues paraprox_stencil_approx on the
     stream given at preparation time."""
 
-    def __init__(self, x, f: Filter, scheme, reach: int, out, *, halo_top=0, halo_bottom=0, stream=None):
+    def __init__(self, x, f: Filter, scheme, reach: int, out, *, halo_top=0, halo_bottom=0, stream=None,
+                 lattice=False):
         _need_cuda(x, out)
         self._img = image_of(x, halo_top, halo_bottom)
         _check_out(out, self._img)
         self._keep = (x, out, f)
         self._args = (f.handle, _scheme(scheme), int(reach), _dp(x, halo_top), _dp(out), C.byref(self._img),
                       _stream(stream))
-        self._fn = _lib.paraprox_stencil_approx
+        self._fn = _lib.paraprox_stencil_lattice if lattice else _lib.paraprox_stencil_approx
 
     def __call__(self):
         rc = self._fn(*self._args)
@@ -381,4 +411,33 @@ def tune_decide(f: Filter, partials, toq: float, metric="mre"):
     sc, rc, q = C.c_int(), C.c_int(), C.c_double()
     _check(_lib.paraprox_tune_decide(f.handle, p.ctypes.data_as(_D) if p.size else None, _metric(metric),
                                      float(toq), C.byref(sc), C.byref(rc), C.byref(q)), "tune_decide")
+    return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+def tune_lattice(frames, f: Filter, toq: float, metric="mre", *, stream=None):
+    """Lattice tuner: returns (scheme name, reach, quality)."""
+    _need_cuda(frames)
+    img = image_of(frames)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune_lattice(f.handle, _dp(frames), C.byref(img), float(toq), _metric(metric),
+                                      C.byref(sc), C.byref(rc), C.byref(q), _stream(stream)), "tune_lattice")
+    return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+def tune_lattice_partials(frames, f: Filter, metric="mre", *, stream=None) -> np.ndarray:
+    _need_cuda(frames)
+    img = image_of(frames)
+    p = np.zeros(12, dtype=np.float64)
+    _check(_lib.paraprox_tune_lattice_partials(f.handle, _dp(frames), C.byref(img), _metric(metric),
+                                               p.ctypes.data_as(_D), _stream(stream)), "tune_lattice_partials")
+    return p
+
+
+def tune_lattice_decide(partials, toq: float, metric="mre"):
+    p = np.ascontiguousarray(partials, dtype=np.float64)
+    if p.size != 12:
+        raise ValueError("12 partials expected")
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune_lattice_decide(p.ctypes.data_as(_D), _metric(metric), float(toq), C.byref(sc),
+                                             C.byref(rc), C.byref(q)), "tune_lattice_decide")
     return SCHEME_NAMES[sc.value], rc.value, q.value
