@@ -53,6 +53,7 @@ extern "C" {
 
 typedef struct CUstream_st* paraprox_stream;       /* == cudaStream_t */
 typedef struct paraprox_filter_s* paraprox_filter; /* opaque, library-owned, immutable */
+typedef struct paraprox_runtime_s* paraprox_runtime; /* opaque, library-owned runtime state */
 
 typedef enum {
     PARAPROX_OK = 0,
@@ -227,6 +228,44 @@ PARAPROX_API paraprox_status paraprox_tune_lattice_partials(paraprox_filter f, c
 PARAPROX_API paraprox_status paraprox_tune_lattice_decide(const double* h_partials12, paraprox_metric m,
                                              double toq, paraprox_scheme* out_scheme, int* out_reach,
                                              double* out_quality);
+
+/* ---- runtime: periodic quality check and back-off (NEXT-2) ------------ */
+
+/* The runtime loop of PAPER.md L572-592 ("checks the output quality
+ * periodically ... If the quality drops below the TOQ, it uses a less
+ * aggressive approximation"; every 40-50 invocations keeps the overhead under
+ * 5 %, L2656-2666).  DESIGN.md readings R1-R4:
+ *  - train: the TOQ tuner on d_train picks rung 0; the ladder continues with
+ *    the later candidates (cost order) whose training quality is higher than
+ *    every earlier rung, and ends at EXACT;
+ *  - run: the current rung's stencil into d_out (asynchronous on s); on the
+ *    1st and then every check_every-th invocation (0 = never) the exact
+ *    stencil of the same input and the quality of d_out against it are also
+ *    enqueued on s, their partials copied to pinned host memory behind an
+ *    event -- the call does not wait for them;
+ *  - a finished check (seen at the next run, or forced by _sync) with quality
+ *    < toq moves one rung down the ladder.
+ * The runtime owns its check buffers (device memory of one output image,
+ * allocated at the first check); the filter must outlive it.  Not for
+ * concurrent use from several threads on different streams (calls are
+ * serialised by a mutex). */
+PARAPROX_API paraprox_status paraprox_runtime_create(paraprox_filter f, double toq, paraprox_metric m,
+                                        int check_every, paraprox_runtime* out);
+PARAPROX_API void paraprox_runtime_destroy(paraprox_runtime rt);
+/* Syncs s. */
+PARAPROX_API paraprox_status paraprox_runtime_train(paraprox_runtime rt, const float* d_train,
+                                       const paraprox_image* img, paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_runtime_run(paraprox_runtime rt, const float* d_in, float* d_out,
+                                     const paraprox_image* img, paraprox_stream s);
+/* Waits for a pending check and applies it. */
+PARAPROX_API paraprox_status paraprox_runtime_sync(paraprox_runtime rt);
+/* Current rung and counters (host-only; any pointer may be NULL). */
+PARAPROX_API paraprox_status paraprox_runtime_state(paraprox_runtime rt, paraprox_scheme* scheme, int* reach,
+                                       long long* invocations, long long* checks, long long* backoffs,
+                                       double* last_quality);
+/* The ladder: *n rungs, at most cap written (arrays may be NULL). */
+PARAPROX_API paraprox_status paraprox_runtime_ladder(paraprox_runtime rt, int cap, int* n,
+                                        paraprox_scheme* schemes, int* reaches, double* train_quality);
 
 /* ---- diagnostics -------------------------------------------------------- */
 

@@ -24,25 +24,21 @@ void count_launch(const char* name) {
     t_last_kernel = name;
 }
 
-static paraprox_status fail(paraprox_status st, const std::string& msg) {
+paraprox_status fail(paraprox_status st, const std::string& msg) {
     t_err = msg;
     return st;
 }
 
-static paraprox_status cuda_fail(cudaError_t e, const char* where) {
+paraprox_status cuda_fail(cudaError_t e, const char* where) {
     t_err = std::string(where) + ": " + cudaGetErrorString(e);
     return e == cudaErrorMemoryAllocation ? PARAPROX_ERR_ALLOC : PARAPROX_ERR_CUDA;
 }
 
-#define PPX_CUDA(call)                                  \
-    do {                                                \
-        cudaError_t _e = (call);                        \
-        if (_e != cudaSuccess) return cuda_fail(_e, #call); \
-    } while (0)
+
 
 static bool odd_k(int k) { return k >= 1 && (k & 1) == 1; }
 
-static paraprox_status check_image(const paraprox_image* img, bool allow_halo) {
+paraprox_status check_image(const paraprox_image* img, bool allow_halo) {
     if (!img) return fail(PARAPROX_ERR_INVALID_ARG, "img is NULL");
     if (img->n < 1 || img->h < 1 || img->w < 1) return fail(PARAPROX_ERR_INVALID_ARG, "n, h, w must be >= 1");
     if (img->pitch < img->w) return fail(PARAPROX_ERR_INVALID_ARG, "pitch < w");
@@ -55,7 +51,7 @@ static paraprox_status check_image(const paraprox_image* img, bool allow_halo) {
     return PARAPROX_OK;
 }
 
-static View view_of(const paraprox_image* img) {
+View view_of(const paraprox_image* img) {
     View v;
     v.n = img->n;
     v.h = img->h;
@@ -68,7 +64,7 @@ static View view_of(const paraprox_image* img) {
 }
 
 // byte ranges touched: inputs (with halos) and outputs must not overlap
-static bool overlaps(const float* in, const float* out, const paraprox_image* img) {
+bool overlaps(const float* in, const float* out, const paraprox_image* img) {
     const long long fs = img->n > 1 ? img->frame_stride : 0;
     const char* i0 = (const char*)(in - (long long)img->halo_top * img->pitch);
     const char* i1 = (const char*)(in + (img->n - 1) * fs + (long long)(img->h - 1 + img->halo_bottom) * img->pitch + img->w);
@@ -77,7 +73,7 @@ static bool overlaps(const float* in, const float* out, const paraprox_image* im
     return i0 < o1 && o0 < i1;
 }
 
-static paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
+paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
                                    const paraprox_image* img, paraprox_stream s) {
     if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
     if (!in || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL buffer");
@@ -113,7 +109,7 @@ static paraprox_status run_lattice(paraprox_filter f, int dy, int dx, const floa
     return PARAPROX_OK;
 }
 
-static double quality_of(const double* p3, paraprox_metric m) {
+double quality_of(const double* p3, paraprox_metric m) {
     if (m == PARAPROX_MRE) return 1.0 - p3[0] / p3[1];
     if (m == PARAPROX_L2) {
         if (p3[1] == 0.0) return p3[0] == 0.0 ? 1.0 : -INFINITY;
@@ -123,12 +119,12 @@ static double quality_of(const double* p3, paraprox_metric m) {
     return mse == 0.0 ? INFINITY : 10.0 * std::log10(255.0 * 255.0 / mse);
 }
 
-static bool metric_ok(paraprox_metric m) { return m == PARAPROX_MRE || m == PARAPROX_L2 || m == PARAPROX_PSNR; }
+bool metric_ok(paraprox_metric m) { return m == PARAPROX_MRE || m == PARAPROX_L2 || m == PARAPROX_PSNR; }
 
 // Stream-ordered scratch comes from a library-owned memory pool per device
 // whose release threshold keeps freed blocks mapped, so repeated calls (the
 // tuner, run_host) do not remap device memory every time.
-static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
     static std::mutex mu;
     static cudaMemPool_t pools[64] = {};
     int dev = 0;
@@ -178,7 +174,7 @@ static paraprox_status quality_partials_impl(const float* e, const float* a, con
 }
 
 // all candidates' partials into h_partials[3 * n]
-static paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
+paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
                                           paraprox_metric m, const std::vector<Candidate>& cands,
                                           double* h_partials, paraprox_stream s) {
     if (!f || !d_train || (!h_partials && !cands.empty())) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
@@ -280,7 +276,7 @@ static paraprox_status decide(const std::vector<Candidate>& cands, const double*
     return PARAPROX_OK;
 }
 
-static paraprox_status check_toq(double toq, paraprox_metric m) {
+paraprox_status check_toq(double toq, paraprox_metric m) {
     if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
     if (m != PARAPROX_PSNR && !(toq > 0.0 && toq <= 1.0)) return fail(PARAPROX_ERR_INVALID_ARG, "toq not in (0, 1]");
     if (std::isnan(toq)) return fail(PARAPROX_ERR_INVALID_ARG, "toq is NaN");

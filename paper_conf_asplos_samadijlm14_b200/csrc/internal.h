@@ -84,6 +84,28 @@ cudaError_t launch_quality(const float* e, const float* a, const View& v, parapr
                            double* d_part3, double* d_scratch, cudaStream_t s);
 constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums
 
+// ---- api.cpp helpers shared with runtime.cpp ----
+#define PPX_CUDA(call)                                  \
+    do {                                                \
+        cudaError_t _e = (call);                        \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call); \
+    } while (0)
+
+paraprox_status fail(paraprox_status st, const std::string& msg);
+paraprox_status cuda_fail(cudaError_t e, const char* where);
+paraprox_status check_image(const paraprox_image* img, bool allow_halo);
+View view_of(const paraprox_image* img);
+bool overlaps(const float* in, const float* out, const paraprox_image* img);
+paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
+                            const paraprox_image* img, paraprox_stream s);
+double quality_of(const double* p3, paraprox_metric m);
+bool metric_ok(paraprox_metric m);
+paraprox_status check_toq(double toq, paraprox_metric m);
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s);
+paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
+                                   paraprox_metric m, const std::vector<Candidate>& cands, double* h_partials,
+                                   paraprox_stream s);
+
 void count_launch(const char* name);
 extern std::atomic<unsigned long long> g_launches;
 extern thread_local const char* t_last_kernel;

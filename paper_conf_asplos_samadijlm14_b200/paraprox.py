@@ -56,6 +56,13 @@ _SIGS = {
     "paraprox_tune_lattice": [_P, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
     "paraprox_tune_lattice_partials": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_tune_lattice_decide": [_D, C.c_int, C.c_double, _I, _I, _D],
+    "paraprox_runtime_create": [_P, C.c_double, C.c_int, C.c_int, C.POINTER(_P)],
+    "paraprox_runtime_train": [_P, _P, _IMG, _P],
+    "paraprox_runtime_run": [_P, _P, _P, _IMG, _P],
+    "paraprox_runtime_sync": [_P],
+    "paraprox_runtime_state": [_P, _I, _I, C.POINTER(C.c_longlong), C.POINTER(C.c_longlong),
+                               C.POINTER(C.c_longlong), _D],
+    "paraprox_runtime_ladder": [_P, C.c_int, _I, _I, _I, _D],
     "paraprox_quality": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials_async": [_P, _P, _IMG, C.c_int, _P, _P],
@@ -70,6 +77,8 @@ for _name, _args in _SIGS.items():
     getattr(_lib, _name).restype = C.c_int
 _lib.paraprox_filter_destroy.argtypes = [_P]
 _lib.paraprox_filter_destroy.restype = None
+_lib.paraprox_runtime_destroy.argtypes = [_P]
+_lib.paraprox_runtime_destroy.restype = None
 _lib.paraprox_status_string.argtypes = [C.c_int]
 _lib.paraprox_status_string.restype = C.c_char_p
 _lib.paraprox_last_error.restype = C.c_char_p
@@ -77,7 +86,7 @@ _lib.paraprox_last_kernel.restype = C.c_char_p
 _lib.paraprox_version.restype = C.c_int
 _lib.paraprox_launch_count.restype = C.c_ulonglong
 
-ABI_SYMBOLS = sorted(list(_SIGS) + ["paraprox_filter_destroy", "paraprox_status_string", "paraprox_last_error",
+ABI_SYMBOLS = sorted(list(_SIGS) + ["paraprox_filter_destroy", "paraprox_runtime_destroy", "paraprox_status_string", "paraprox_last_error",
                                     "paraprox_last_kernel", "paraprox_version", "paraprox_launch_count"])
 
 
@@ -441,3 +450,64 @@ def tune_lattice_decide(partials, toq: float, metric="mre"):
     _check(_lib.paraprox_tune_lattice_decide(p.ctypes.data_as(_D), _metric(metric), float(toq), C.byref(sc),
                                              C.byref(rc), C.byref(q)), "tune_lattice_decide")
     return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+class Runtime:
+    """The runtime loop (paraprox_runtime_*): train once, then run the current
+    rung; every ``check_every``-th invocation is checked against the exact
+    stencil on the device and a quality below ``toq`` moves one rung down the
+    ladder."""
+
+    def __init__(self, f: Filter, toq: float, metric="mre", check_every: int = 40):
+        self._f = f
+        h = _P()
+        _check(_lib.paraprox_runtime_create(f.handle, float(toq), _metric(metric), int(check_every), C.byref(h)),
+               "runtime_create")
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            _lib.paraprox_runtime_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def train(self, frames, *, stream=None):
+        _need_cuda(frames)
+        img = image_of(frames)
+        _check(_lib.paraprox_runtime_train(self._h, _dp(frames), C.byref(img), _stream(stream)), "runtime_train")
+        return self.state()
+
+    def run(self, x, out=None, *, halo_top=0, halo_bottom=0, stream=None):
+        _need_cuda(x)
+        img = image_of(x, halo_top, halo_bottom)
+        out = _out_like(x, halo_top, halo_bottom, out)
+        _need_cuda(out)
+        _check_out(out, img)
+        _check(_lib.paraprox_runtime_run(self._h, _dp(x, halo_top), _dp(out), C.byref(img), _stream(stream)),
+               "runtime_run")
+        return out
+
+    def sync(self):
+        _check(_lib.paraprox_runtime_sync(self._h), "runtime_sync")
+
+    def state(self):
+        sc, r = C.c_int(), C.c_int()
+        inv, chk, bo = C.c_longlong(), C.c_longlong(), C.c_longlong()
+        q = C.c_double()
+        _check(_lib.paraprox_runtime_state(self._h, C.byref(sc), C.byref(r), C.byref(inv), C.byref(chk),
+                                           C.byref(bo), C.byref(q)), "runtime_state")
+        return dict(scheme=SCHEME_NAMES[sc.value], reach=r.value, invocations=inv.value, checks=chk.value,
+                    backoffs=bo.value, last_quality=q.value)
+
+    def ladder(self):
+        n = C.c_int()
+        _check(_lib.paraprox_runtime_ladder(self._h, 0, C.byref(n), None, None, None), "runtime_ladder")
+        k = max(1, n.value)
+        s, r, q = (C.c_int * k)(), (C.c_int * k)(), (C.c_double * k)()
+        _check(_lib.paraprox_runtime_ladder(self._h, k, C.byref(n), s, r, q), "runtime_ladder")
+        return [(SCHEME_NAMES[s[i]], r[i], q[i]) for i in range(n.value)]

@@ -171,3 +171,23 @@ def test_device_calls_refuse_cpu_tensors(P):
     f = P.Filter(F.gaussian(3))
     with pytest.raises(TypeError):
         P.stencil_exact(torch.zeros(8, 8), f)
+
+
+def test_runtime_argument_errors(P):
+    import ctypes as C
+    from workloads import filters as F
+    f = P.Filter(F.mean(5))
+    h = C.c_void_p()
+    assert P._lib.paraprox_runtime_create(f.handle, 1.5, P.MRE, 40, C.byref(h)) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_runtime_create(f.handle, 0.9, P.MRE, -1, C.byref(h)) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_runtime_create(None, 0.9, P.MRE, 40, C.byref(h)) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_runtime_create(f.handle, 0.9, P.MRE, 40, C.byref(h)) == P.OK
+    img = P.Image(1, 8, 8, 8, 64, 0, 0)
+    # untrained: refused before any device work
+    assert P._lib.paraprox_runtime_run(h, None, None, C.byref(img), None) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_runtime_state(h, None, None, None, None, None, None) == P.ERR_INVALID_ARG
+    n = C.c_int()
+    assert P._lib.paraprox_runtime_ladder(h, 0, C.byref(n), None, None, None) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_runtime_sync(h) == P.OK
+    P._lib.paraprox_runtime_destroy(h)
+    P._lib.paraprox_runtime_destroy(None)

@@ -1,0 +1,125 @@
+"""GPU tests of the runtime loop (NEXT-2; PAPER.md L572-592, L2656-2666;
+DESIGN.md R1-R4): ladder construction, outputs equal to the stencil of the
+current rung, periodic device-side checks, back-off on a quality drop, and
+the check overhead at the paper's 1-in-40 rate."""
+import numpy as np
+import pytest
+import torch
+
+import workloads as W
+from workloads import filters as F
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def P():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_asplos_samadijlm14_b200 as pkg
+
+    return pkg.paraprox
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+@pytest.mark.parametrize("name,w,metric", [("gauss3", F.gaussian(3), "mre"), ("mean5", F.mean(5), "mre"),
+                                           ("conv9", F.conv(9), "l2"), ("sep7", F.separable(7), "l2")])
+def test_ladder(P, O, name, w, metric):
+    f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+    train = dev(W.frames(4, 192, 256, 0))
+    for toq in (0.80, 0.90, 0.95, 0.99):
+        rt = P.Runtime(f, toq, metric, check_every=10)
+        st = rt.train(train)
+        lad = rt.ladder()
+        assert (st["scheme"], st["reach"]) == P.tune(train, f, toq, metric)[:2]  # R1: rung 0 = the tuner
+        assert lad[-1][:2] == ("exact", 0)                                        # R2 ends at exact
+        qs = [q for _, _, q in lad]
+        assert all(a < b for a, b in zip(qs, qs[1:])), lad                       # strictly less aggressive
+        if lad[0][0] != "exact":
+            assert qs[0] >= toq
+        order = P.tune_candidates(f)
+        idx = [order.index(r[:2]) for r in lad[:-1]]
+        assert idx == sorted(idx)                                                 # cost order kept
+        rt.close()
+
+
+def test_outputs_and_checks(P, O):
+    f = P.Filter(F.mean(5))
+    train = dev(W.frames(4, 256, 256, 0))
+    frames = dev(W.frames(12, 256, 256, 20))
+    rt = P.Runtime(f, 0.9, "mre", check_every=4)
+    st = rt.train(train)
+    out = torch.empty_like(frames[0:1])
+    for k in range(12):
+        before = rt.state()
+        rt.run(frames[k:k + 1], out=out)
+        ref = P.stencil_approx(frames[k:k + 1], f, before["scheme"], before["reach"])
+        assert torch.equal(out, ref), k
+        if k % 4 == 0:  # a checked invocation: the check measures exactly this output
+            rt.sync()
+            q = P.quality(P.stencil_exact(frames[k:k + 1], f), out, "mre")
+            assert rt.state()["last_quality"] == pytest.approx(q, abs=1e-12)
+    s = rt.state()
+    assert s["invocations"] == 12 and s["checks"] == 3 and s["backoffs"] == 0
+    assert (s["scheme"], s["reach"]) == (st["scheme"], st["reach"])
+
+
+def test_backoff_to_exact_on_noise(P):
+    f = P.Filter(F.mean(5))
+    rt = P.Runtime(f, 0.9, "mre", check_every=1)
+    rt.train(dev(W.frames(4, 128, 128, 0)))
+    lad = rt.ladder()
+    assert len(lad) >= 2
+    # a checkerboard breaks the adjacent-similarity assumption:
+    # every approximate rung misses the TOQ on it
+    yy, xx = np.mgrid[0:128, 0:128]
+    noise = dev((16.0 + 219.0 * ((yy + xx) % 2)).astype(np.float32)[None])
+    out = torch.empty_like(noise)
+    seen = []
+    for _ in range(len(lad) + 3):
+        rt.run(noise, out=out)
+        rt.sync()
+        s = rt.state()
+        seen.append((s["scheme"], s["reach"]))
+    assert seen[-1] == ("exact", 0)
+    assert rt.state()["backoffs"] == len(lad) - 1
+    # every rung was visited in ladder order
+    assert [r[:2] for r in lad[1:]] == [x for i, x in enumerate(seen) if i == 0 or x != seen[i - 1]][:len(lad) - 1]
+    checks = rt.state()["checks"]
+    rt.run(noise, out=out)
+    rt.sync()
+    assert rt.state()["checks"] == checks  # exact is never checked
+    assert torch.equal(out, P.stencil_exact(noise, f))
+
+
+def test_check_overhead_at_one_in_forty(P):
+    """a check every 40-50 invocations costs < 5 %.  Reported;
+    asserted loosely (shared boxes are noisy)."""
+    f = P.Filter(F.mean(5))
+    train = dev(W.frames(2, 1024, 1024, 0))
+    x = torch.rand(8, 2048, 2048, device="cuda") * 8 + 120  # 128 MiB in + out: larger than L2
+    out = torch.empty_like(x)
+
+    def timed(every):
+        rt = P.Runtime(f, 0.9, "mre", check_every=every)
+        rt.train(train)
+        for _ in range(5):
+            rt.run(x, out=out)
+        rt.sync()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record()
+        for _ in range(200):
+            rt.run(x, out=out)
+        e1.record()
+        torch.cuda.synchronize()
+        rt.sync()
+        return e0.elapsed_time(e1)
+
+    runs = [(timed(0), timed(40)) for _ in range(3)]  # interleaved
+    base = min(b for b, _ in runs)
+    chk = min(c for _, c in runs)
+    print(f"runtime overhead at 1/40 checks: {100 * (chk / base - 1):.2f} %  ({base:.3f} ms -> {chk:.3f} ms)")
+    assert chk / base < 1.15

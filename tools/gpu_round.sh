@@ -7,10 +7,10 @@ timeout 900 python -m pytest tests -m gpu -q --maxfail=30 ${PYTEST_K:+-k "$PYTES
 tail -3 gpurun_out/pytest_gpu.log
 timeout 300 python bench.py > gpurun_out/bench_c2.json 2> gpurun_out/bench_c2.err; echo bench rc=$?
 for c in c1 c3 c4; do
-  timeout 300 python bench.py --workload $c --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 2 > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; echo bench $c rc=$?
+  timeout 400 python bench.py --workload $c --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 2 > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; echo bench $c rc=$?
 done
 if [ -z "$NO_NCU" ]; then
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_c2.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 1 > gpurun_out/ncu_launches.log 2>&1; echo ncu-launches rc=$?
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_tiles -c 6 -o gpurun_out/prof_c2 -f python tools/prof_run.py --workload c2 --schemes exact:0,center:2,row:1 --reps 2 > gpurun_out/ncu_c2.log 2>&1; echo ncu rc=$?
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 600 --csv --log-file gpurun_out/launches_c2.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --e2e-steps 1 > gpurun_out/ncu_launches.log 2>&1; echo ncu-launches rc=$?
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_tiles|k_pointwise|k_lattice|k_quality_flat" -c 12 -o gpurun_out/prof_c2 -f python tools/prof_run.py --workload c2 --schemes exact:0,center:2,row:1 --lattice row:1,row:4 --quality --reps 2 > gpurun_out/ncu_c2.log 2>&1; echo ncu rc=$?
 fi
 cat gpurun_out/bench_c2.json

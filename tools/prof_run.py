@@ -16,6 +16,7 @@ def main():
     ap.add_argument("--schemes", default="exact:0,center:2")
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quality", action="store_true")
+    ap.add_argument("--lattice", default="", help="lattice schemes, e.g. row:1,row:4")
     args = ap.parse_args()
     import torch
 
@@ -48,6 +49,12 @@ def main():
         if args.quality:
             for _ in range(args.reps):
                 P.quality(e, out, wl["metric"])
+    for spec in filter(None, args.lattice.split(",")):
+        s, r = spec.split(":")
+        for _ in range(args.reps):
+            P.stencil_lattice(x, f, s, int(r), out=out)
+        torch.cuda.synchronize()
+        print("lattice", spec, P.last_kernel())
 
 
 if __name__ == "__main__":
