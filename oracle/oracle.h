@@ -28,7 +28,8 @@ extern "C" {
 
 /* schemes and metrics use the oracle's own numbering (same meaning as the
  * library's, defined independently) */
-enum { OR_EXACT = 0, OR_ROW = 1, OR_COL = 2, OR_CENTER = 3 };
+enum { OR_EXACT = 0, OR_ROW = 1, OR_COL = 2, OR_CENTER = 3,
+       OR_SKIP_ROW = 4, OR_SKIP_COL = 5, OR_SKIP_BOTH = 6 /* reduction approximation */ };
 enum { OR_MRE = 0, OR_L2 = 1, OR_PSNR = 2 };
 
 /* Reaching-distance rule for one axis of a tile of radius r (PAPER.md
@@ -105,6 +106,26 @@ int oracle_tune_lattice(const float* x, int n, int h, int w, int separable,
                         const float* wgt_or_wy, int ky, const float* wx, int kx,
                         double toq, int metric, double* qualities4,
                         int* scheme, int* reach, double* quality);
+
+/* Reduction approximation of the stencil loops (§3.3.3;
+ * NEXT-3): the filter-row loop executes every ny-th iteration from its first
+ * (i = -r_y, -r_y+ny, ...) and the filter-column loop every nx-th, each loop
+ * summing into a zero-initialised temporary that is multiplied by its
+ * skipping rate after the loop.  Rates above the trip count saturate to it.
+ * Schemes: skip-row (N, 1), skip-col (1, N), skip-both (N, N). */
+int oracle_scheme_skips(int scheme, int rate, int* ny, int* nx);
+int oracle_stencil_skip(const float* x, int n, int h, int w, const float* wgt, int ky, int kx,
+                        int ny, int nx, double* out);
+int oracle_stencil_skip_sep(const float* x, int n, int h, int w, const float* wy, int ky,
+                            const float* wx, int kx, int ny, int nx, double* out);
+
+/* Extended tuner: flags bit 0 = stencil schemes, bit 1 = reduction schemes
+ * (rates 2..r+1), one cost order over both (O7 + S24). */
+int oracle_tune_candidates_ex(int ky, int kx, int separable, int flags, int cap, int* schemes, int* rates);
+int oracle_tune_ex(const float* x, int n, int h, int w, int separable,
+                   const float* wgt_or_wy, int ky, const float* wx, int kx, int flags,
+                   double toq, int metric, int cap, double* qualities,
+                   int* n_evaluated, int* scheme, int* rate, double* quality);
 
 #ifdef __cplusplus
 }

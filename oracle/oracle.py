@@ -18,10 +18,13 @@ _HDR = os.path.join(_HERE, "oracle.h")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 EXACT, ROW, COL, CENTER = 0, 1, 2, 3
+SKIP_ROW, SKIP_COL, SKIP_BOTH = 4, 5, 6
 MRE, L2, PSNR = 0, 1, 2
-SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "center": CENTER, "centre": CENTER}
+SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "center": CENTER, "centre": CENTER,
+           "skip_row": SKIP_ROW, "skip_col": SKIP_COL, "skip_both": SKIP_BOTH}
 METRICS = {"mre": MRE, "l2": L2, "psnr": PSNR}
-SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center"}
+SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center", SKIP_ROW: "skip_row",
+                SKIP_COL: "skip_col", SKIP_BOTH: "skip_both"}
 
 
 def build(force: bool = False) -> str:
@@ -63,7 +66,16 @@ def lib():
                                      C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
         _lib.oracle_tune_lattice.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
                                              C.c_double, C.c_int, f64, i32, i32, f64]
-        for name in ("oracle_tune_lattice", "oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
+        _lib.oracle_scheme_skips.argtypes = [C.c_int, C.c_int, i32, i32]
+        _lib.oracle_stencil_skip.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, C.c_int,
+                                             C.c_int, C.c_int, f64]
+        _lib.oracle_stencil_skip_sep.argtypes = [f32, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                                 C.c_int, C.c_int, f64]
+        _lib.oracle_tune_candidates_ex.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_int, i32, i32]
+        _lib.oracle_tune_ex.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
+                                        C.c_int, C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
+        for name in ("oracle_scheme_skips", "oracle_stencil_skip", "oracle_stencil_skip_sep",
+                     "oracle_tune_candidates_ex", "oracle_tune_ex", "oracle_tune_lattice", "oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
                      "oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
                      "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
                      "oracle_tune_candidates", "oracle_tune"):
@@ -246,3 +258,73 @@ def tune_lattice(x, w, toq: float, metric="mre"):
     _ok(lib().oracle_tune_lattice(_fp(x), n, h, ww, sep, _fp(wa), ky, _fp(wb), kx, float(toq), m, _dp(qs),
                                   C.byref(sc), C.byref(rc), C.byref(q)), "tune_lattice")
     return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value, qualities=[float(v) for v in qs])
+
+
+def stencil_skip_xy(x, w, ny: int, nx: int) -> np.ndarray:
+    """Reduction approximation of the stencil loops:
+    every ny-th filter row / nx-th filter column, each loop scaled by its rate.
+    ``w`` is a 2-D array (dense) or a (wy, wx) pair (separable)."""
+    x, squeeze = _frames(x)
+    out = np.empty(x.shape, dtype=np.float64)
+    n, h, ww = x.shape
+    if isinstance(w, (tuple, list)):
+        wy = np.ascontiguousarray(w[0], dtype=np.float32).ravel()
+        wx = np.ascontiguousarray(w[1], dtype=np.float32).ravel()
+        _ok(lib().oracle_stencil_skip_sep(_fp(x), n, h, ww, _fp(wy), wy.size, _fp(wx), wx.size, ny, nx, _dp(out)),
+            "stencil_skip_sep")
+    else:
+        w = np.ascontiguousarray(w, dtype=np.float32)
+        _ok(lib().oracle_stencil_skip(_fp(x), n, h, ww, _fp(w), w.shape[0], w.shape[1], ny, nx, _dp(out)),
+            "stencil_skip")
+    return out[0] if squeeze else out
+
+
+def scheme_skips(scheme, rate: int):
+    ny, nx = C.c_int(), C.c_int()
+    s = SCHEMES[scheme] if isinstance(scheme, str) else int(scheme)
+    _ok(lib().oracle_scheme_skips(s, int(rate), C.byref(ny), C.byref(nx)), "scheme_skips")
+    return ny.value, nx.value
+
+
+def stencil_scheme(x, w, scheme, reach: int) -> np.ndarray:
+    """Any scheme of the library (stencil or reduction), dense or separable."""
+    s = SCHEMES[scheme] if isinstance(scheme, str) else int(scheme)
+    if s >= SKIP_ROW:
+        return stencil_skip_xy(x, w, *scheme_skips(s, reach))
+    if isinstance(w, (tuple, list)):
+        return stencil_sep_scheme(x, w[0], w[1], s, reach)
+    return stencil_approx(x, w, s, reach)
+
+
+def tune_candidates_ex(ky: int, kx: int, separable: bool = False, flags: int = 3):
+    cap = 128
+    s = np.zeros(cap, dtype=np.int32)
+    r = np.zeros(cap, dtype=np.int32)
+    n = lib().oracle_tune_candidates_ex(ky, kx, int(separable), int(flags), cap,
+                                        s.ctypes.data_as(C.POINTER(C.c_int)), r.ctypes.data_as(C.POINTER(C.c_int)))
+    if n < 0:
+        raise ValueError("tune_candidates_ex rejected its arguments")
+    return [(SCHEME_NAMES[int(s[i])], int(r[i])) for i in range(n)]
+
+
+def tune_ex(x, w, toq: float, metric="mre", flags: int = 3, all_qualities: bool = False):
+    """Extended oracle tuner over stencil (bit 0) and reduction (bit 1) schemes."""
+    x, _ = _frames(x)
+    m = METRICS[metric] if isinstance(metric, str) else int(metric)
+    n, h, ww = x.shape
+    if isinstance(w, (tuple, list)):
+        wa = np.ascontiguousarray(w[0], dtype=np.float32).ravel()
+        wb = np.ascontiguousarray(w[1], dtype=np.float32).ravel()
+        sep, ky, kx = 1, wa.size, wb.size
+    else:
+        wa = np.ascontiguousarray(w, dtype=np.float32)
+        sep, ky, kx, wb = 0, wa.shape[0], wa.shape[1], wa
+    cap = 128
+    qs = np.full(cap, np.nan)
+    nev, sc, rc = C.c_int(), C.c_int(), C.c_int()
+    q = C.c_double()
+    _ok(lib().oracle_tune_ex(_fp(x), n, h, ww, sep, _fp(wa), ky, _fp(wb), kx, int(flags), float(toq), m, cap,
+                             _dp(qs) if all_qualities else None, C.byref(nev), C.byref(sc), C.byref(rc),
+                             C.byref(q)), "tune_ex")
+    return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value,
+                qualities=[float(v) for v in qs[:nev.value]] if all_qualities else None)
