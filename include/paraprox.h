@@ -65,12 +65,21 @@ typedef enum {
 } paraprox_status;
 
 /* Fig. 6 (L1156-1166): exact; row (rows within the reach copy the accessed
- * row); column; centre (the tile centre stands in for its neighbours). */
+ * row); column; centre (the tile centre stands in for its neighbours).
+ * The reduction approximation of the stencil's loops (§3.3.3,
+ * applied to Convolution Separable's loops, L1920-1996; NEXT-3): skip-row
+ * executes every N-th filter row (the vertical loop) and scales by N,
+ * skip-col every N-th filter column, skip-both both loops; with these schemes
+ * the "reach" argument is the skipping rate N >= 1 (1 = exact; rates above
+ * the loop's trip count saturate to it). */
 typedef enum {
     PARAPROX_EXACT = 0,
     PARAPROX_ROW = 1,
     PARAPROX_COL = 2,
-    PARAPROX_CENTER = 3
+    PARAPROX_CENTER = 3,
+    PARAPROX_SKIP_ROW = 4,
+    PARAPROX_SKIP_COL = 5,
+    PARAPROX_SKIP_BOTH = 6
 } paraprox_scheme;
 
 /* Table 1 (L1644-1664): mean relative error (Gaussian, mean filters) and
@@ -147,6 +156,14 @@ PARAPROX_API paraprox_status paraprox_stencil_lattice_xy(paraprox_filter f, int 
                                             const float* d_in, float* d_out,
                                             const paraprox_image* img, paraprox_stream s);
 
+/* Reduction approximation with per-loop skipping rates (skip_y, skip_x >= 1;
+ * rates above the loop's trip count saturate): every skip_y-th filter row
+ * and skip_x-th filter column from the first, each loop scaled by its rate
+ * (§3.3.3).  (1, 1) is the exact stencil. */
+PARAPROX_API paraprox_status paraprox_stencil_skip_xy(paraprox_filter f, int skip_y, int skip_x,
+                                         const float* d_in, float* d_out,
+                                         const paraprox_image* img, paraprox_stream s);
+
 /* End-to-end convenience over HOST buffers: copies h_in to the device,
  * runs the stencil (scheme, reach), copies the result to h_out, overlapping
  * the transfers with the kernels chunk by chunk.  Pinned host memory gives
@@ -212,6 +229,24 @@ PARAPROX_API paraprox_status paraprox_tune_partials(paraprox_filter f, const flo
 PARAPROX_API paraprox_status paraprox_tune_decide(paraprox_filter f, const double* h_partials,
                                      paraprox_metric m, double toq, paraprox_scheme* out_scheme,
                                      int* out_reach, double* out_quality);
+
+/* Extended tuner over the stencil schemes (flags bit 0) and the reduction
+ * schemes (flags bit 1: skip-both / skip-row / skip-col with rates 2..r+1),
+ * one integer cost order over both (O7 + S24).  flags = 1 is
+ * paraprox_tune.  Same conventions as the functions above; the returned
+ * "reach" is the skipping rate for the reduction schemes. */
+PARAPROX_API paraprox_status paraprox_tune_ex(paraprox_filter f, int flags, const float* d_train,
+                                 const paraprox_image* img, double toq, paraprox_metric m,
+                                 paraprox_scheme* out_scheme, int* out_reach, double* out_quality,
+                                 paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_tune_candidates_ex(paraprox_filter f, int flags, int cap, int* n,
+                                            paraprox_scheme* schemes, int* reaches);
+PARAPROX_API paraprox_status paraprox_tune_partials_ex(paraprox_filter f, int flags, const float* d_train,
+                                          const paraprox_image* img, paraprox_metric m,
+                                          double* h_partials, paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_tune_decide_ex(paraprox_filter f, int flags, const double* h_partials,
+                                        paraprox_metric m, double toq, paraprox_scheme* out_scheme,
+                                        int* out_reach, double* out_quality);
 
 /* Lattice tuner: the exact stencil once on d_train, then the row lattice
  * with reach 4, 3, 2, 1 (fewest HBM bytes first); the first whose quality

@@ -73,20 +73,47 @@ bool overlaps(const float* in, const float* out, const paraprox_image* img) {
     return i0 < o1 && o0 < i1;
 }
 
-paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
-                                   const paraprox_image* img, paraprox_stream s) {
+// skip = false: (a, b) are reaches (dy, dx); skip = true: skipping rates (sy, sx)
+static paraprox_status run_plan(paraprox_filter f, bool skip, int a, int b, const float* in, float* out,
+                                const paraprox_image* img, paraprox_stream s) {
     if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
     if (!in || !out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL buffer");
-    if (dy < 0 || dx < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    if (!skip && (a < 0 || b < 0)) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    if (skip && (a < 1 || b < 1)) return fail(PARAPROX_ERR_INVALID_ARG, "skipping rate < 1");
     paraprox_status st = check_image(img, true);
     if (st != PARAPROX_OK) return st;
     if (overlaps(in, out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_in");
-    const Plan& p = get_plan(f, dy, dx);
+    const Plan& p = skip ? get_plan_skip(f, a, b) : get_plan(f, a, b);
     const View v = view_of(img);
     const long long ofs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
     cudaError_t e = launch_stencil(p, in, v, out, img->pitch, ofs, (cudaStream_t)s);
     if (e != cudaSuccess) return cuda_fail(e, "stencil launch");
     return PARAPROX_OK;
+}
+
+paraprox_status run_stencil(paraprox_filter f, int dy, int dx, const float* in, float* out,
+                            const paraprox_image* img, paraprox_stream s) {
+    return run_plan(f, false, dy, dx, in, out, img, s);
+}
+
+// any scheme, stencil (reach) or reduction (skipping rate)
+static paraprox_status run_scheme(paraprox_filter f, paraprox_scheme scheme, int reach, const float* in, float* out,
+                                  const paraprox_image* img, paraprox_stream s) {
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_SKIP_BOTH) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (is_skip_scheme(scheme)) {
+        if (reach < 1) return fail(PARAPROX_ERR_INVALID_ARG, "skipping rate < 1");
+        int sy, sx;
+        scheme_skips(scheme, reach, &sy, &sx);
+        return run_plan(f, true, sy, sx, in, out, img, s);
+    }
+    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    return run_plan(f, false, dy, dx, in, out, img, s);
+}
+
+static const Plan& cand_plan(paraprox_filter f, const Candidate& c) {
+    return is_skip_scheme(c.scheme) ? get_plan_skip(f, c.dy, c.dx) : get_plan(f, c.dy, c.dx);
 }
 
 constexpr int kMaxLatticeReach = 1 << 20;
@@ -206,7 +233,7 @@ paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, cons
     cudaError_t e = launch_stencil(get_plan(f, 0, 0), d_train, vin, E, img->w, plane, cs);
     if (e != cudaSuccess) return cuda_fail(e, "exact launch");
     for (size_t k = 0; k < nc; ++k) {
-        e = launch_stencil(get_plan(f, cands[k].dy, cands[k].dx), d_train, vin, A, img->w, plane, cs);
+        e = launch_stencil(cand_plan(f, cands[k]), d_train, vin, A, img->w, plane, cs);
         if (e != cudaSuccess) return cuda_fail(e, "candidate launch");
         e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);
         if (e != cudaSuccess) return cuda_fail(e, "quality launch");
@@ -349,11 +376,12 @@ paraprox_status paraprox_stencil_exact(paraprox_filter f, const float* d_in, flo
 
 paraprox_status paraprox_stencil_approx(paraprox_filter f, paraprox_scheme scheme, int reach, const float* d_in,
                                         float* d_out, const paraprox_image* img, paraprox_stream s) {
-    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
-    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
-    int dy, dx;
-    scheme_reaches(scheme, reach, &dy, &dx);
-    return run_stencil(f, dy, dx, d_in, d_out, img, s);
+    return run_scheme(f, scheme, reach, d_in, d_out, img, s);
+}
+
+paraprox_status paraprox_stencil_skip_xy(paraprox_filter f, int skip_y, int skip_x, const float* d_in, float* d_out,
+                                         const paraprox_image* img, paraprox_stream s) {
+    return run_plan(f, true, skip_y, skip_x, d_in, d_out, img, s);
 }
 
 paraprox_status paraprox_stencil_approx_xy(paraprox_filter f, int reach_y, int reach_x, const float* d_in,
@@ -463,6 +491,54 @@ paraprox_status paraprox_tune_candidates(paraprox_filter f, int cap, int* n, par
     return PARAPROX_OK;
 }
 
+paraprox_status paraprox_tune_candidates_ex(paraprox_filter f, int flags, int cap, int* n, paraprox_scheme* schemes,
+                                            int* reaches) {
+    if (!f || !n) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (cap < 0) return fail(PARAPROX_ERR_INVALID_ARG, "cap < 0");
+    if (flags < 1 || flags > 3) return fail(PARAPROX_ERR_INVALID_ARG, "flags not in 1..3");
+    std::vector<Candidate> c = candidates_ex(f, flags);
+    *n = (int)c.size();
+    for (int k = 0; k < (int)c.size() && k < cap; ++k) {
+        if (schemes) schemes[k] = c[k].scheme;
+        if (reaches) reaches[k] = c[k].reach;
+    }
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_tune_partials_ex(paraprox_filter f, int flags, const float* d_train,
+                                          const paraprox_image* img, paraprox_metric m, double* h_partials,
+                                          paraprox_stream s) {
+    if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
+    if (flags < 1 || flags > 3) return fail(PARAPROX_ERR_INVALID_ARG, "flags not in 1..3");
+    return tune_partials_impl(f, d_train, img, m, candidates_ex(f, flags), h_partials, s);
+}
+
+paraprox_status paraprox_tune_decide_ex(paraprox_filter f, int flags, const double* h_partials, paraprox_metric m,
+                                        double toq, paraprox_scheme* out_scheme, int* out_reach,
+                                        double* out_quality) {
+    if (!f || !out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (flags < 1 || flags > 3) return fail(PARAPROX_ERR_INVALID_ARG, "flags not in 1..3");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    std::vector<Candidate> c = candidates_ex(f, flags);
+    if (!h_partials && !c.empty()) return fail(PARAPROX_ERR_INVALID_ARG, "NULL partials");
+    return decide(c, h_partials, m, toq, out_scheme, out_reach, out_quality);
+}
+
+paraprox_status paraprox_tune_ex(paraprox_filter f, int flags, const float* d_train, const paraprox_image* img,
+                                 double toq, paraprox_metric m, paraprox_scheme* out_scheme, int* out_reach,
+                                 double* out_quality, paraprox_stream s) {
+    if (!f || !out_scheme || !out_reach || !out_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (flags < 1 || flags > 3) return fail(PARAPROX_ERR_INVALID_ARG, "flags not in 1..3");
+    paraprox_status st = check_toq(toq, m);
+    if (st != PARAPROX_OK) return st;
+    std::vector<Candidate> c = candidates_ex(f, flags);
+    std::vector<double> parts(3 * c.size() + 3);
+    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s);
+    if (st != PARAPROX_OK) return st;
+    return decide(c, parts.data(), m, toq, out_scheme, out_reach, out_quality);
+}
+
 paraprox_status paraprox_tune_partials(paraprox_filter f, const float* d_train, const paraprox_image* img,
                                        paraprox_metric m, double* h_partials, paraprox_stream s) {
     if (!f) return fail(PARAPROX_ERR_INVALID_ARG, "filter is NULL");
@@ -495,14 +571,15 @@ paraprox_status paraprox_tune(paraprox_filter f, const float* d_train, const par
 paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int reach, const float* h_in,
                                   float* h_out, const paraprox_image* img, paraprox_stream s) {
     if (!f || !h_in || !h_out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
-    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
-    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_SKIP_BOTH) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < (is_skip_scheme(scheme) ? 1 : 0)) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0 or rate < 1");
     paraprox_status st = check_image(img, false);
     if (st != PARAPROX_OK) return st;
     if (overlaps(h_in, h_out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "h_out overlaps h_in");
     int dy, dx;
-    scheme_reaches(scheme, reach, &dy, &dx);
-    const Plan& p = get_plan(f, dy, dx);
+    if (is_skip_scheme(scheme)) scheme_skips(scheme, reach, &dy, &dx);
+    else scheme_reaches(scheme, reach, &dy, &dx);
+    const Plan& p = is_skip_scheme(scheme) ? get_plan_skip(f, dy, dx) : get_plan(f, dy, dx);
     cudaStream_t cs = (cudaStream_t)s;
     const int n = img->n, h = img->h, w = img->w;
     const long long plane = (long long)h * w;

@@ -28,6 +28,7 @@ void register_r1_sep();
 void register_r2_sep();
 void register_r3_sep();
 void register_r4_sep();
+void register_r8_sep();
 
 namespace {
 
@@ -58,6 +59,7 @@ void init_registry() {
         register_r2_sep();
         register_r3_sep();
         register_r4_sep();
+        register_r8_sep();
     });
 }
 
@@ -127,8 +129,8 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.ofs = ofs;
     TapW W = {};
     if (p.separable) {
-        for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 4] = p.wyf[i];
-        for (int j = 0; j < p.nx; ++j) W.wx[p.ax[j] + 4] = p.wxf[j];
+        for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 8] = p.wyf[i];
+        for (int j = 0; j < p.nx; ++j) W.wx[p.ax[j] + 8] = p.wxf[j];
     } else {
         for (int i = 0; i < p.ny; ++i)
             for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];
@@ -156,7 +158,8 @@ cudaError_t launch_stencil(const Plan& p, const float* in, const View& v, float*
                            long long ofs, cudaStream_t s) {
     // a plan that accesses only the centre is a map: stream it (k_pointwise.cu)
     if (!force_generic() && p.hy == 0 && p.hx == 0) return launch_pointwise(p, in, v, out, opitch, ofs, s);
-    if (!force_generic() && p.ry <= 4 && p.rx <= 4) {
+    const int rmax = p.separable ? 8 : 4;  // tile instances: dense r <= 4, separable r <= 8
+    if (!force_generic() && p.ry <= rmax && p.rx <= rmax) {
         init_registry();
         for (Entry& e : reg()) {
             if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;

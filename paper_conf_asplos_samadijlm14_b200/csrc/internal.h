@@ -26,6 +26,7 @@ struct Plan {
     int ky = 1, kx = 1, ry = 0, rx = 0;
     bool separable = false;
     int dy = 0, dx = 0;                 // reaches, saturated to the radius
+    int sy = 1, sx = 1;                 // reduction skipping rates (1 = none), saturated to K
     int my[kMaxK] = {}, mx[kMaxK] = {}; // index maps, m[i + r]
     int ny = 0, nx = 0;                 // |Ry|, |Rx| accessed offsets per axis
     int ay[kMaxK] = {}, ax[kMaxK] = {}; // accessed offsets, ascending
@@ -61,6 +62,13 @@ namespace ppx {
 // ---- plan.cpp ----
 int map_offset(int r, int d, int i);
 const Plan& get_plan(paraprox_filter f, int dy, int dx);
+// reduction approximation of the filter loops (§3.3.3): every sy-th
+// filter row and sx-th filter column from the first, weights scaled by the rates
+const Plan& get_plan_skip(paraprox_filter f, int sy, int sx);
+bool is_skip_scheme(paraprox_scheme s);
+void scheme_skips(paraprox_scheme s, int rate, int* sy, int* sx);
+// candidates of the extended tuner: flags bit 0 stencil schemes, bit 1 reduction schemes
+std::vector<Candidate> candidates_ex(paraprox_filter f, int flags);
 void scheme_reaches(paraprox_scheme s, int reach, int* dy, int* dx);
 std::vector<Candidate> candidates(paraprox_filter f);
 

@@ -114,7 +114,7 @@ __device__ __forceinline__ void block_sum2(double& s0, double& s1) {
 constexpr int kQU = 4;
 
 template <int M>
-__global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
+__global__ void __launch_bounds__(256, 4) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
                                                       long long count, double* __restrict__ part) {
     QAcc<M> q;
     const long long n4 = count >> 2;
@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ 
 }
 
 template <int M>
-__global__ void __launch_bounds__(256) k_quality_partials(const float* __restrict__ E,
+__global__ void __launch_bounds__(256, 4) k_quality_partials(const float* __restrict__ E,
                                                           const float* __restrict__ A, View v,
                                                           double* __restrict__ part) {
     QAcc<M> q;

@@ -40,9 +40,9 @@ constexpr int kTH = kRB * kWarps;        // 64 tile rows
 constexpr int kThreads = 32 * kWarps;
 
 struct TapW {
-    float w[9][9];   // dense folded weights at [a + 4][b + 4]
-    float wy[9];     // separable folded weights at [a + 4]
-    float wx[9];
+    float w[9][9];   // dense folded weights at [a + 4][b + 4]   (r <= 4)
+    float wy[17];    // separable folded weights at [a + 8]     (r <= 8)
+    float wx[17];
 };
 
 struct TileArgs {
@@ -238,7 +238,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
                     hz[q][0] = hz[q][1] = make_float2(0.f, 0.f);
                     static_for<2 * HX + 1>([&](auto B) {
                         constexpr int b = decltype(B)::value - HX;
-                        if constexpr (has(MASKX, b)) fma_pairs<NV, HXP + b>(hz[q], W.wx[b + 4], ve, vo);
+                        if constexpr (has(MASKX, b)) fma_pairs<NV, HXP + b>(hz[q], W.wx[b + 8], ve, vo);
                     });
                 }
             }
@@ -261,7 +261,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
                 for (int k = 0; k < kRB; ++k) {
                     const int a = rr - HY - k;
                     if (a < -HY || a > HY || !has(MASKY, a)) continue;
-                    const float wt = W.wy[a + 4];
+                    const float wt = W.wy[a + 8];
                     const float2 w2 = make_float2(wt, wt);
                     acc[k][0] = __ffma2_rn(w2, t0, acc[k][0]);
                     acc[k][1] = __ffma2_rn(w2, t1, acc[k][1]);

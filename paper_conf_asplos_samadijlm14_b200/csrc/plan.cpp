@@ -96,6 +96,69 @@ static Plan make_plan(const paraprox_filter_s& f, int dy, int dx) {
     return p;
 }
 
+// PAPER.md §3.3.3 (L1366-1404): "Paraprox multiplies the loop step by N ...
+// inserts adjustment code after the loop.  This code multiplies the result by
+// the skipping rate".  Applied to the filter-row loop (rate sy) and the
+// filter-column loop (rate sx): the executed offsets are -r, -r+s, ... <= r,
+// and each executed weight is scaled by the rates (fp64 product, one fp32
+// rounding).  Rates above the trip count K saturate to K (reading S24).
+static void build_skip_axis(int r, int s, int* m, int* reps, int* nrep, int* halo, uint32_t* mask) {
+    for (int i = -r; i <= r; ++i) m[i + r] = i;
+    *nrep = 0;
+    *halo = 0;
+    *mask = 0;
+    for (int a = -r; a <= r; a += s) {
+        reps[(*nrep)++] = a;
+        *halo = std::max(*halo, std::abs(a));
+        *mask |= 1u << (a + kMaxR);
+    }
+}
+
+static Plan make_plan_skip(const paraprox_filter_s& f, int sy, int sx) {
+    Plan p;
+    p.ky = f.ky;
+    p.kx = f.kx;
+    p.ry = f.ky / 2;
+    p.rx = f.kx / 2;
+    p.separable = f.separable;
+    p.sy = std::min(sy, f.ky);
+    p.sx = std::min(sx, f.kx);
+    build_skip_axis(p.ry, p.sy, p.my, p.ay, &p.ny, &p.hy, &p.masky);
+    build_skip_axis(p.rx, p.sx, p.mx, p.ax, &p.nx, &p.hx, &p.maskx);
+    if (f.separable) {
+        for (int k = 0; k < p.ny; ++k) p.wyf[k] = (float)((double)p.sy * (double)f.wy[p.ay[k] + p.ry]);
+        for (int k = 0; k < p.nx; ++k) p.wxf[k] = (float)((double)p.sx * (double)f.wx[p.ax[k] + p.rx]);
+        p.taps = p.ny + p.nx;
+    } else {
+        for (int a = 0; a < p.ny; ++a)
+            for (int b = 0; b < p.nx; ++b)
+                p.wf[a * p.nx + b] = (float)((double)p.sy * (double)p.sx *
+                                             (double)f.w[(p.ay[a] + p.ry) * f.kx + (p.ax[b] + p.rx)]);
+        p.taps = p.ny * p.nx;
+    }
+    return p;
+}
+
+const Plan& get_plan_skip(paraprox_filter f, int sy, int sx) {
+    sy = std::min(std::max(sy, 1), f->ky);
+    sx = std::min(std::max(sx, 1), f->kx);
+    if (sy == 1 && sx == 1) return get_plan(f, 0, 0);
+    std::lock_guard<std::mutex> lk(f->mu);
+    auto key = std::make_pair(-sy, -sx);  // reach keys are >= 0
+    auto it = f->plans.find(key);
+    if (it == f->plans.end()) it = f->plans.emplace(key, make_plan_skip(*f, sy, sx)).first;
+    return it->second;
+}
+
+bool is_skip_scheme(paraprox_scheme s) {
+    return s == PARAPROX_SKIP_ROW || s == PARAPROX_SKIP_COL || s == PARAPROX_SKIP_BOTH;
+}
+
+void scheme_skips(paraprox_scheme s, int rate, int* sy, int* sx) {
+    *sy = (s == PARAPROX_SKIP_ROW || s == PARAPROX_SKIP_BOTH) ? rate : 1;
+    *sx = (s == PARAPROX_SKIP_COL || s == PARAPROX_SKIP_BOTH) ? rate : 1;
+}
+
 const Plan& get_plan(paraprox_filter f, int dy, int dx) {
     dy = std::min(dy, f->ky / 2);
     dx = std::min(dx, f->kx / 2);
@@ -149,6 +212,57 @@ std::vector<Candidate> candidates(paraprox_filter f) {
         if (!dup) out.push_back(c);
     }
     return out;
+}
+
+}  // namespace ppx
+
+namespace ppx {
+
+// The extended tuner's candidates (reading S24): the stencil candidates above
+// (flags bit 0) and the reduction schemes (bit 1) -- skip-both, skip-row,
+// skip-col with rate N in 2..r+1 of the skipped axis (skip-both: the smaller
+// radius), offered only on axes with r >= 1 -- in one order by the integer
+// cost key (taps, hy, hx, scheme id: centre 0, row 1, col 2, skip-both 3,
+// skip-row 4, skip-col 5, rate); a reduction candidate whose saturated rates
+// equal an earlier one's is dropped.
+std::vector<Candidate> candidates_ex(paraprox_filter f, int flags) {
+    std::vector<Candidate> all;
+    if (flags & 1) all = candidates(f);
+    if (flags & 2) {
+        const int ry = f->ky / 2, rx = f->kx / 2;
+        const paraprox_scheme fam[3] = {PARAPROX_SKIP_BOTH, PARAPROX_SKIP_ROW, PARAPROX_SKIP_COL};
+        std::vector<Candidate> sk;
+        for (int q = 0; q < 3; ++q) {
+            const int rmax = fam[q] == PARAPROX_SKIP_ROW ? ry : fam[q] == PARAPROX_SKIP_COL ? rx : std::min(ry, rx);
+            if (rmax < 1) continue;
+            for (int n = 2; n <= rmax + 1; ++n) {
+                Candidate c;
+                c.scheme = fam[q];
+                c.reach = n;
+                int sy, sx;
+                scheme_skips(c.scheme, n, &sy, &sx);
+                const Plan& p = get_plan_skip(f, sy, sx);
+                c.dy = p.sy;  // for skip candidates dy/dx carry the saturated rates
+                c.dx = p.sx;
+                c.taps = p.taps;
+                c.hy = p.hy;
+                c.hx = p.hx;
+                c.sid = 3 + q;
+                bool dup = false;
+                for (const Candidate& o : sk) dup = dup || (o.dy == c.dy && o.dx == c.dx);
+                if (!dup) sk.push_back(c);
+            }
+        }
+        all.insert(all.end(), sk.begin(), sk.end());
+    }
+    std::stable_sort(all.begin(), all.end(), [](const Candidate& a, const Candidate& b) {
+        if (a.taps != b.taps) return a.taps < b.taps;
+        if (a.hy != b.hy) return a.hy < b.hy;
+        if (a.hx != b.hx) return a.hx < b.hx;
+        if (a.sid != b.sid) return a.sid < b.sid;
+        return a.reach < b.reach;
+    });
+    return all;
 }
 
 }  // namespace ppx

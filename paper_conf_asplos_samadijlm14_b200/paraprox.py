@@ -25,9 +25,12 @@ _lib = C.CDLL(LIB_PATH)
 
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CUDA, ERR_ALLOC = range(5)
 EXACT, ROW, COL, CENTER = 0, 1, 2, 3
+SKIP_ROW, SKIP_COL, SKIP_BOTH = 4, 5, 6
 MRE, L2, PSNR = 0, 1, 2
-SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "column": COL, "center": CENTER, "centre": CENTER}
-SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center"}
+SCHEMES = {"exact": EXACT, "row": ROW, "col": COL, "column": COL, "center": CENTER, "centre": CENTER,
+           "skip_row": SKIP_ROW, "skip_col": SKIP_COL, "skip_both": SKIP_BOTH}
+SCHEME_NAMES = {EXACT: "exact", ROW: "row", COL: "col", CENTER: "center", SKIP_ROW: "skip_row",
+                SKIP_COL: "skip_col", SKIP_BOTH: "skip_both"}
 METRICS = {"mre": MRE, "l2": L2, "psnr": PSNR}
 MAX_K = 17
 
@@ -52,6 +55,11 @@ _SIGS = {
     "paraprox_stencil_approx_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_run_host": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_stencil_lattice": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_stencil_skip_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_tune_ex": [_P, C.c_int, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
+    "paraprox_tune_candidates_ex": [_P, C.c_int, C.c_int, _I, _I, _I],
+    "paraprox_tune_partials_ex": [_P, C.c_int, _P, _IMG, C.c_int, _D, _P],
+    "paraprox_tune_decide_ex": [_P, C.c_int, _D, C.c_int, C.c_double, _I, _I, _D],
     "paraprox_stencil_lattice_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_tune_lattice": [_P, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
     "paraprox_tune_lattice_partials": [_P, _P, _IMG, C.c_int, _D, _P],
@@ -301,6 +309,19 @@ def stencil_lattice_xy(x, f: Filter, reach_y: int, reach_x: int, out=None, *, st
     return out
 
 
+def stencil_skip_xy(x, f: Filter, skip_y: int, skip_x: int, out=None, *, halo_top=0, halo_bottom=0, stream=None):
+    """Reduction approximation of the filter loops: every
+    skip_y-th filter row / skip_x-th filter column, scaled by the rates."""
+    _need_cuda(x)
+    img = image_of(x, halo_top, halo_bottom)
+    out = _out_like(x, halo_top, halo_bottom, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_skip_xy(f.handle, int(skip_y), int(skip_x), _dp(x, halo_top), _dp(out),
+                                         C.byref(img), _stream(stream)), "stencil_skip_xy")
+    return out
+
+
 class Prepared:
     """A stencil call with its arguments marshalled once (for tight loops and
     graph capture): calling it re-issues paraprox_stencil_approx on the
@@ -511,3 +532,45 @@ class Runtime:
         s, r, q = (C.c_int * k)(), (C.c_int * k)(), (C.c_double * k)()
         _check(_lib.paraprox_runtime_ladder(self._h, k, C.byref(n), s, r, q), "runtime_ladder")
         return [(SCHEME_NAMES[s[i]], r[i], q[i]) for i in range(n.value)]
+
+
+STENCIL, REDUCTION = 1, 2  # tune_ex flags
+
+
+def tune_candidates_ex(f: Filter, flags: int = 3):
+    n = C.c_int()
+    _check(_lib.paraprox_tune_candidates_ex(f.handle, int(flags), 0, C.byref(n), None, None), "tune_candidates_ex")
+    s = (C.c_int * max(1, n.value))()
+    r = (C.c_int * max(1, n.value))()
+    _check(_lib.paraprox_tune_candidates_ex(f.handle, int(flags), n.value, C.byref(n), s, r), "tune_candidates_ex")
+    return [(SCHEME_NAMES[s[i]], r[i]) for i in range(n.value)]
+
+
+def tune_ex(frames, f: Filter, toq: float, metric="mre", flags: int = 3, *, stream=None):
+    """Extended tuner over stencil (flags & 1) and reduction (flags & 2)
+    schemes.  Returns (scheme name, reach or skipping rate, quality)."""
+    _need_cuda(frames)
+    img = image_of(frames)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune_ex(f.handle, int(flags), _dp(frames), C.byref(img), float(toq), _metric(metric),
+                                 C.byref(sc), C.byref(rc), C.byref(q), _stream(stream)), "tune_ex")
+    return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+def tune_partials_ex(frames, f: Filter, metric="mre", flags: int = 3, *, stream=None) -> np.ndarray:
+    _need_cuda(frames)
+    img = image_of(frames)
+    n = len(tune_candidates_ex(f, flags))
+    p = np.zeros(3 * max(n, 1), dtype=np.float64)
+    _check(_lib.paraprox_tune_partials_ex(f.handle, int(flags), _dp(frames), C.byref(img), _metric(metric),
+                                          p.ctypes.data_as(_D), _stream(stream)), "tune_partials_ex")
+    return p[:3 * n]
+
+
+def tune_decide_ex(f: Filter, partials, toq: float, metric="mre", flags: int = 3):
+    p = np.ascontiguousarray(partials, dtype=np.float64)
+    sc, rc, q = C.c_int(), C.c_int(), C.c_double()
+    _check(_lib.paraprox_tune_decide_ex(f.handle, int(flags), p.ctypes.data_as(_D) if p.size else None,
+                                        _metric(metric), float(toq), C.byref(sc), C.byref(rc), C.byref(q)),
+           "tune_decide_ex")
+    return SCHEME_NAMES[sc.value], rc.value, q.value

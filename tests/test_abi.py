@@ -191,3 +191,32 @@ def test_runtime_argument_errors(P):
     assert P._lib.paraprox_runtime_sync(h) == P.OK
     P._lib.paraprox_runtime_destroy(h)
     P._lib.paraprox_runtime_destroy(None)
+
+
+@pytest.mark.parametrize("ky,kx", [(1, 1), (1, 5), (3, 3), (5, 5), (3, 7), (9, 9), (9, 1), (17, 17), (15, 3)])
+@pytest.mark.parametrize("sep", [False, True])
+@pytest.mark.parametrize("flags", [1, 2, 3])
+def test_candidates_ex_match_oracle(P, O, ky, kx, sep, flags):
+    rng = np.random.default_rng(ky * 31 + kx)
+    if sep:
+        f = P.Filter(wy=rng.uniform(0, 1, ky).astype(np.float32), wx=rng.uniform(0, 1, kx).astype(np.float32))
+    else:
+        f = P.Filter(rng.uniform(0, 1, (ky, kx)).astype(np.float32))
+    assert P.tune_candidates_ex(f, flags) == O.tune_candidates_ex(ky, kx, sep, flags)
+    if flags == 1:
+        assert P.tune_candidates_ex(f, 1) == P.tune_candidates(f)
+
+
+def test_skip_argument_errors(P):
+    import ctypes as C
+    from workloads import filters as F
+    f = P.Filter(F.mean(5))
+    img = P.Image(1, 8, 8, 8, 64, 0, 0)
+    buf = C.c_void_p(16)
+    out = C.c_void_p(1 << 20)
+    assert P._lib.paraprox_stencil_skip_xy(f.handle, 0, 1, buf, out, C.byref(img), None) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_stencil_approx(f.handle, P.SKIP_ROW, 0, buf, out, C.byref(img), None) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_stencil_approx(f.handle, 7, 1, buf, out, C.byref(img), None) == P.ERR_INVALID_ARG
+    n = C.c_int()
+    assert P._lib.paraprox_tune_candidates_ex(f.handle, 0, 0, C.byref(n), None, None) == P.ERR_INVALID_ARG
+    assert P._lib.paraprox_tune_candidates_ex(f.handle, 4, 0, C.byref(n), None, None) == P.ERR_INVALID_ARG

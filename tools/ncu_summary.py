@@ -42,6 +42,14 @@ def short(name):
     if m:
         sep = m.group(5) in ("1", "true")
         return f"{'sep' if sep else 'dense'}_{SETS.get(int(m.group(3)), m.group(3))}_{SETS.get(int(m.group(4)), m.group(4))}"
+    m = re.match(r"void (?:ppx::)?k_pointwise_(flat|rows)<(\d|true|false)>", name)
+    if m:
+        kind = "sep" if m.group(2) in ("1", "true") else "dense"
+        return f"{kind}_map" + ("_rows" if m.group(1) == "rows" else "")
+    m = re.match(r"void (?:ppx::)?k_lattice<(\d+), (\d+), (\d|true|false)>", name)
+    if m:
+        kind = "sep" if m.group(3) in ("1", "true") else "dense"
+        return f"lattice_{kind}_s{m.group(1)}_r{m.group(2)}"
     m = re.match(r"void (?:ppx::)?(\w+)(<[^>]*>)?", name)
     return (m.group(1) + (m.group(2) or "")) if m else name[:70]
 
