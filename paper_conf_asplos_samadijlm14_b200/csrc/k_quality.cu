@@ -21,6 +21,8 @@ namespace ppx {
 template <int M>
 struct QAcc {
     double s0 = 0.0, s1 = 0.0;
+    bool bad = false;                                       // never set: no fix-up pass
+    __device__ __forceinline__ void fix(float, float) {}
     __device__ __forceinline__ void add(float e, float a) {
         const double de = (double)e, da = (double)a;
         const double d = da - de;
@@ -52,30 +54,37 @@ __device__ __forceinline__ float rcp_approx(float x) {
 template <>
 struct QAcc<PARAPROX_MRE> {
     double hi = 0.0, lo = 0.0;  // sums of the leading and trailing parts of the terms
-    __device__ __forceinline__ void add_slow(float e, float a) {
-        const double de = (double)e, da = (double)a;
-        const double q = de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
-        hi += q;
+    bool bad = false;  // a term the pair arithmetic cannot carry was skipped
+    // the fast path skips terms with |E| tiny or huge or |A-E| huge (and the
+    // E == 0 convention, S12); a second pass adds exactly those in fp64
+    __device__ __forceinline__ static bool fast_ok(float ae, float dh) {
+        return ae >= 1e-30f && ae <= 1e30f && fabsf(dh) <= 1e30f;
     }
     __device__ __forceinline__ void add(float e, float a) {
         float dh, dl;
         two_sum(a, -e, dh, dl);  // A - E exactly, as dh + dl
         const float ae = fabsf(e);
-        if (ae >= 1e-30f && ae <= 1e30f && fabsf(dh) <= 1e30f) {
-            if (dh < 0.f) {
-                dh = -dh;
-                dl = -dl;
-            }
-            // q0 + q1 = |A-E| / |E| to ~2^-46: the remainder of the first
-            // quotient is exact under the FMA, so the approximate reciprocal's
-            // own error is corrected by the second term
-            const float rc = rcp_approx(ae);
-            const float q0 = __fmul_rn(dh, rc);
-            const float rem = __fadd_rn(__fmaf_rn(-q0, ae, dh), dl);
-            hi += (double)q0;
-            lo += (double)__fmul_rn(rem, rc);
-        } else {  // rare: fp64 quotient (or the E == 0 convention, S12)
-            add_slow(e, a);
+        const bool ok = fast_ok(ae, dh);
+        bad |= !ok;
+        if (dh < 0.f) {
+            dh = -dh;
+            dl = -dl;
+        }
+        // q0 + q1 = |A-E| / |E| to ~2^-46: the remainder of the first quotient
+        // is exact under the FMA, so the approximate reciprocal's own error is
+        // corrected by the second term
+        const float rc = rcp_approx(ae);
+        const float q0 = __fmul_rn(dh, rc);
+        const float rem = __fadd_rn(__fmaf_rn(-q0, ae, dh), dl);
+        hi += ok ? (double)q0 : 0.0;
+        lo += ok ? (double)__fmul_rn(rem, rc) : 0.0;
+    }
+    __device__ __forceinline__ void fix(float e, float a) {
+        float dh, dl;
+        two_sum(a, -e, dh, dl);
+        if (!fast_ok(fabsf(e), dh)) {
+            const double de = (double)e, da = (double)a;
+            hi += de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
         }
     }
     __device__ __forceinline__ void get(double& a, double& b) const {
@@ -114,35 +123,41 @@ __device__ __forceinline__ void block_sum2(double& s0, double& s1) {
 constexpr int kQU = 4;
 
 template <int M>
-__global__ void __launch_bounds__(256, 4) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
+__global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
                                                       long long count, double* __restrict__ part) {
     QAcc<M> q;
     const long long n4 = count >> 2;
     const long long stride = (long long)gridDim.x * blockDim.x;
     const float4* e4 = reinterpret_cast<const float4*>(E);
     const float4* a4 = reinterpret_cast<const float4*>(A);
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kQU * stride) {
-        float4 e[kQU], a[kQU];
+    auto sweep = [&](auto&& op) {
+        for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kQU * stride) {
+            float4 e[kQU], a[kQU];
 #pragma unroll
-        for (int u = 0; u < kQU; ++u) {
-            const long long j = i + u * stride;
-            if (j < n4) {
-                e[u] = __ldcs(e4 + j);
-                a[u] = __ldcs(a4 + j);
-            } else {
-                e[u] = a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int u = 0; u < kQU; ++u) {
+                const long long j = i + u * stride;
+                if (j < n4) {
+                    e[u] = __ldcs(e4 + j);
+                    a[u] = __ldcs(a4 + j);
+                } else {
+                    e[u] = a[u] = make_float4(1.f, 1.f, 1.f, 1.f);  // |1-1|/|1| = 0, (1-1)^2 = 0
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kQU; ++u) {
+                if (i + u * stride >= n4) continue;
+                op(e[u].x, a[u].x);
+                op(e[u].y, a[u].y);
+                op(e[u].z, a[u].z);
+                op(e[u].w, a[u].w);
             }
         }
-#pragma unroll
-        for (int u = 0; u < kQU; ++u) {
-            q.add(e[u].x, a[u].x);
-            q.add(e[u].y, a[u].y);
-            q.add(e[u].z, a[u].z);
-            q.add(e[u].w, a[u].w);
-        }
-    }
-    if (blockIdx.x == 0)
-        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) q.add(E[x], A[x]);
+        if (blockIdx.x == 0)
+            for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) op(E[x], A[x]);
+    };
+    sweep([&](float e, float a) { q.add(e, a); });
+    if constexpr (M == PARAPROX_MRE)
+        if (__syncthreads_or(q.bad)) sweep([&](float e, float a) { q.fix(e, a); });
     double s0, s1;
     q.get(s0, s1);
     block_sum2(s0, s1);
@@ -153,7 +168,7 @@ __global__ void __launch_bounds__(256, 4) k_quality_flat(const float* __restrict
 }
 
 template <int M>
-__global__ void __launch_bounds__(256, 4) k_quality_partials(const float* __restrict__ E,
+__global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_partials(const float* __restrict__ E,
                                                           const float* __restrict__ A, View v,
                                                           double* __restrict__ part) {
     QAcc<M> q;
@@ -161,34 +176,39 @@ __global__ void __launch_bounds__(256, 4) k_quality_partials(const float* __rest
     const bool vec = ((v.pitch & 3) == 0) && ((v.fstride & 3) == 0) &&
                      ((((uintptr_t)E) | ((uintptr_t)A)) & 15) == 0;
     const int w4 = vec ? (v.w >> 2) : 0;
-    for (long long R = blockIdx.x; R < rows; R += gridDim.x) {
-        const long long f = R / v.h, y = R - f * v.h;
-        const long long off = f * v.fstride + y * v.pitch;
-        const float4* e4 = reinterpret_cast<const float4*>(E + off);
-        const float4* a4 = reinterpret_cast<const float4*>(A + off);
-        for (int x = threadIdx.x; x < w4; x += kQU * blockDim.x) {
-            float4 e[kQU], a[kQU];
+    auto sweep = [&](auto&& op) {
+        for (long long R = blockIdx.x; R < rows; R += gridDim.x) {
+            const long long f = R / v.h, y = R - f * v.h;
+            const long long off = f * v.fstride + y * v.pitch;
+            const float4* e4 = reinterpret_cast<const float4*>(E + off);
+            const float4* a4 = reinterpret_cast<const float4*>(A + off);
+            for (int x = threadIdx.x; x < w4; x += kQU * blockDim.x) {
+                float4 e[kQU], a[kQU];
 #pragma unroll
-            for (int u = 0; u < kQU; ++u) {
-                const int j = x + u * blockDim.x;
-                if (j < w4) {
-                    e[u] = __ldcs(e4 + j);
-                    a[u] = __ldcs(a4 + j);
-                } else {
-                    e[u] = a[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int u = 0; u < kQU; ++u) {
+                    const int j = x + u * blockDim.x;
+                    if (j < w4) {
+                        e[u] = __ldcs(e4 + j);
+                        a[u] = __ldcs(a4 + j);
+                    } else {
+                        e[u] = a[u] = make_float4(1.f, 1.f, 1.f, 1.f);
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < kQU; ++u) {
+                    if (x + u * (int)blockDim.x >= w4) continue;
+                    op(e[u].x, a[u].x);
+                    op(e[u].y, a[u].y);
+                    op(e[u].z, a[u].z);
+                    op(e[u].w, a[u].w);
                 }
             }
-#pragma unroll
-            for (int u = 0; u < kQU; ++u) {
-                q.add(e[u].x, a[u].x);
-                q.add(e[u].y, a[u].y);
-                q.add(e[u].z, a[u].z);
-                q.add(e[u].w, a[u].w);
-            }
+            for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x) op(__ldcs(E + off + x), __ldcs(A + off + x));
         }
-        for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x)
-            q.add(__ldcs(E + off + x), __ldcs(A + off + x));
-    }
+    };
+    sweep([&](float e, float a) { q.add(e, a); });
+    if constexpr (M == PARAPROX_MRE)
+        if (__syncthreads_or(q.bad)) sweep([&](float e, float a) { q.fix(e, a); });
     double s0, s1;
     q.get(s0, s1);
     block_sum2(s0, s1);
