@@ -172,8 +172,15 @@ def dist_setup():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if ws > 1:
         import torch.distributed as dist
+        # one process per GPU; PARAPROX_DIST_BACKEND=gloo exercises the same
+        # code path with several ranks sharing a device (tests on 1-GPU boxes)
+        local = local % max(1, torch.cuda.device_count())
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("PARAPROX_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
         return dist, rank, ws, local
     return None, 0, 1, local
 
@@ -230,6 +237,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-lattice", action="store_true")
+    ap.add_argument("--no-graph", action="store_true", help="time the eager ctypes loop instead of CUDA graphs")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -323,14 +331,76 @@ def main():
     def exact_step(k):
         exact_ops[k % nbuf]()
 
+    # CUDA graphs: the launch-bound loop (c2 kernels run ~20 us) is captured
+    # once -- G launches rotating over the buffers, G a multiple of nbuf so
+    # consecutive launches never reuse a buffer -- and replayed; exactly K
+    # launches run in the timed region (R replays of G plus one graph of the
+    # remainder).  The eager loop (one ctypes call per launch) is timed too.
+    G = nbuf * max(1, 32 // nbuf)
+
+    class GraphLoop:
+        def __init__(self, make_ops, counts):
+            self.s = torch.cuda.Stream(device=dev)
+            self.ops = make_ops(self.s)
+            with torch.cuda.stream(self.s):
+                for k in range(2 * nbuf):
+                    self.ops[k % nbuf]()
+            torch.cuda.synchronize()
+            self.graphs = {}
+            for n in {G} | {c % G for c in counts if c % G}:
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=self.s):
+                    for k in range(n):
+                        self.ops[k % nbuf]()
+                self.graphs[n] = g
+            torch.cuda.synchronize()
+
+        def run(self, steps):
+            r, rem = divmod(steps, G)
+            for _ in range(r):
+                self.graphs[G].replay()
+            if rem:
+                self.graphs[rem].replay()
+
+    def timed_graph(loop, steps, warmup):
+        loop.run(warmup)
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0.record(stream)
+        loop.run(steps)
+        t1.record(stream)
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        tot = torch.tensor([t0.elapsed_time(t1)], device=dev, dtype=torch.float64)
+        if dist:
+            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        return float(tot[0]), float(tot[0]) / steps, steps  # one kernel node per step
+
     def copy_step(k):  # context: torch's own device copy of the same bytes
         outputs[k % nbuf].copy_(inputs[k % nbuf])
 
-    with ClockSampler(local) as clk:
-        total_ms, kern_ms, launches = timed(approx_step, args.steps, args.warmup)
+    counts = (args.steps, args.warmup)
+    if not args.no_graph:
+        approx_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, scheme, reach, outputs[k], stream=st)
+                                            for k in range(nbuf)], counts)
         approx_kernel = P.last_kernel()
-        exact_total_ms, exact_kern_ms, _ = timed(exact_step, args.steps, args.warmup)
+        exact_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, "exact", 0, outputs[k], stream=st)
+                                           for k in range(nbuf)], counts)
         exact_kernel = P.last_kernel()
+    with ClockSampler(local) as clk:
+        eager_total_ms, eager_kern_ms, eager_launches = timed(approx_step, args.steps, args.warmup)
+        if args.no_graph:
+            approx_kernel = P.last_kernel()
+            total_ms, kern_ms, launches = eager_total_ms, eager_kern_ms, eager_launches
+            exact_total_ms, exact_kern_ms, _ = timed(exact_step, args.steps, args.warmup)
+            exact_kernel = P.last_kernel()
+        else:
+            total_ms, kern_ms, launches = timed_graph(approx_loop, args.steps, args.warmup)
+            exact_total_ms, exact_kern_ms, _ = timed_graph(exact_loop, args.steps, args.warmup)
         copy_ms, _, _ = timed(copy_step, args.steps, args.warmup)
 
         # a4: the quality reduction alone (exact vs approx buffers, 8 B/px read)
@@ -353,9 +423,14 @@ def main():
                 l_scheme, l_reach, l_q = P.tune_lattice(train_keep, f, args.toq, wl["metric"])
             lat = {"scheme": l_scheme, "reach": l_reach, "quality_train": l_q}
             if l_scheme != "exact":
-                lat_ops = [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=stream, lattice=True)
-                           for k in range(nbuf)]
-                lat_total, lat_kern, _ = timed(lambda k: lat_ops[k % nbuf](), args.steps, args.warmup)
+                if args.no_graph:
+                    lat_ops = [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=stream, lattice=True)
+                               for k in range(nbuf)]
+                    lat_total, lat_kern, _ = timed(lambda k: lat_ops[k % nbuf](), args.steps, args.warmup)
+                else:
+                    lat_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=st,
+                                                               lattice=True) for k in range(nbuf)], counts)
+                    lat_total, lat_kern, _ = timed_graph(lat_loop, args.steps, args.warmup)
                 lat_bpp = 4.0 / (2 * l_reach + 1) + 4.0
                 lat.update({
                     "kernel": P.last_kernel(), "ms_per_step": lat_total / args.steps,
@@ -412,9 +487,33 @@ def main():
         if dist:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t[0]) / args.e2e_steps
+        # context: pinned H2D and D2H of the same bytes at once on two streams
+        # (the bound of an overlapped host round trip)
+        hb = torch.empty(px_step, dtype=torch.float32, pin_memory=True)
+        db = torch.empty(px_step, dtype=torch.float32, device=dev)
+        db2 = torch.empty(px_step, dtype=torch.float32, device=dev)
+        s_up, s_dn = torch.cuda.Stream(device=dev), torch.cuda.Stream(device=dev)
+        hb2 = torch.empty(px_step, dtype=torch.float32, pin_memory=True)
+
+        def duplex():
+            with torch.cuda.stream(s_up):
+                db.copy_(hb, non_blocking=True)
+            with torch.cuda.stream(s_dn):
+                hb2.copy_(db2, non_blocking=True)
+            torch.cuda.synchronize()
+
+        duplex()
+        t0 = time.perf_counter()
+        for _ in range(3):
+            duplex()
+        duplex_gbs = 4 * px_step / ((time.perf_counter() - t0) / 3) / 1e9
+        del hb, hb2, db, db2
         e2e = {"value": px_step * ws / e2e_s / 1e6, "unit": "Mpixel/s", "h2d_bytes_per_step": 4 * px_step,
                "d2h_bytes_per_step": 4 * px_step, "steps": args.e2e_steps,
                "api": "paraprox_run_host (pinned host in/out; H2D, kernel, D2H overlapped in chunks)",
+               "pcie_duplex_gbs_each_way": duplex_gbs,
+               "bound_mpx_s": duplex_gbs * 1e9 / 4 / 1e6 * ws,
+               "frac_of_pcie_bound": (px_step * ws / e2e_s / 1e6) / (duplex_gbs * 1e9 / 4 / 1e6 * ws),
                "timing": "host wall clock around synchronous calls, max over ranks"}
         del hin, hout
 
@@ -455,6 +554,8 @@ def main():
                       "kernel_gbs": exact_achieved, "roofline_frac": exact_achieved / peak, "kernel": exact_kernel},
             "copy_same_bytes_gbs": alg_bytes * args.steps / (copy_ms * 1e-3) / 1e9,
             "speedup_vs_exact": exact_ms_step / ms_step,
+            "launch_mode": "eager" if args.no_graph else f"cuda_graph ({G} launches per graph, replayed)",
+            "eager_ms_per_step": eager_total_ms / args.steps,
             "quality_kernel": {"metric": wl["metric"], "ms": qual_kern_ms, "kernel": "quality_flat",
                                "achieved_gbs": alg_bytes / (qual_kern_ms * 1e-3) / 1e9,
                                "frac": alg_bytes / (qual_kern_ms * 1e-3) / 1e9 / peak,

@@ -590,7 +590,10 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     float* din = (float*)buf.p;
     float* dout = din + plane * n;
     // chunks: frames when batched, else row bands (halo rows come along)
-    const int chunks = n > 1 ? std::min(n, 8) : std::max(1, std::min(8, h / 512));
+    // ~4 MiB per chunk (fill and drain of the copy pipeline are one chunk each), at most 32
+    const long long total_bytes = (long long)sizeof(float) * plane * n;
+    const int want = (int)std::min<long long>(32, std::max<long long>(1, total_bytes >> 22));
+    const int chunks = n > 1 ? std::min(n, want) : std::max(1, std::min(want, h / 64));
     cudaStream_t up = nullptr, down = nullptr;
     PPX_CUDA(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
     cudaError_t err = cudaStreamCreateWithFlags(&down, cudaStreamNonBlocking);
