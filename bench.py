@@ -226,6 +226,91 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def run_stripes(args, dist, rank, ws, local):
+    """Config c4 at N > 1 (BASELINE.json configs[3]): one 32768^2 image split
+    into row stripes, one per rank, with the halo rows the plan needs (h_y)
+    exchanged with the two neighbours by NCCL send/recv each step, overlapped
+    with the interior rows (dist.stencil_stripe).  Strong scaling: the whole
+    image is the work at every N."""
+    import torch
+    import paper_conf_asplos_samadijlm14_b200 as pkg
+    from paper_conf_asplos_samadijlm14_b200 import dist as D
+    import workloads as W
+    P = pkg.paraprox
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    wl = WORKLOADS["c4"]
+    kind, w = make_filter_arrays(wl["filter"])
+    f = P.Filter(w)
+    h, wd = wl["h"], wl["w"]
+    r = w.shape[0] // 2
+    s = D.stripe_of(h, ws, rank, cap=r)
+    tile = W.image(4096, 4096, 10)  # the global image is this tile repeated (seamless, periodic)
+    rows = np.tile(tile[np.arange(s.r0 - s.halo_top(r), s.r1 + s.halo_bottom(r)) % 4096], (1, wd // 4096))
+    buf = D.alloc_stripe(s, wd, device=dev)
+    c0 = s.cap - s.halo_top(r)
+    buf[c0:c0 + rows.shape[0]].copy_(torch.from_numpy(rows))
+    out = torch.empty((s.rows, wd), device=dev)
+    train = torch.from_numpy(W.frames(2, 4096, 4096, 1000 * rank)).to(dev)
+    t0 = time.perf_counter()
+    pt = torch.from_numpy(P.tune_partials(train, f, wl["metric"])).to(dev)
+    dist.all_reduce(pt)
+    scheme, reach, q_train = P.tune_decide(f, pt.cpu().numpy(), args.toq, wl["metric"])
+    tune_ms = 1e3 * (time.perf_counter() - t0)
+    del train
+    dy, dx = {"exact": (0, 0), "row": (reach, 0), "col": (0, reach), "center": (reach, reach)}[scheme]
+    hy = f.plan_info(dy, dx)["halo_y"]
+
+    def timed(step):
+        for _ in range(args.warmup):
+            step()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        dist.barrier()
+        torch.cuda.synchronize()
+        l0 = P.launch_count()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        dist.barrier()
+        launches = P.launch_count() - l0
+        tot = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        return float(tot[0]) / args.steps, launches
+
+    with ClockSampler(local) as clk:
+        ms, launches = timed(lambda: D.stencil_stripe(buf, s, f, scheme, reach, out))
+        approx_kernel = P.last_kernel()
+        ex_ms, _ = timed(lambda: D.stencil_stripe(buf, s, f, "exact", 0, out))
+    peak, peak_kind = load_peaks()
+    local_bytes = 8.0 * s.rows * wd
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": h * wd / (ms * 1e-3) / 1e6, "unit": "Mpixel/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "c4", "desc": wl["desc"] + ", row stripes", "h": h, "w": wd, "filter": "conv9",
+                       "toq": args.toq, "metric_quality": wl["metric"],
+                       "parallelism": f"row stripes x{ws}: {s.rows} rows per rank, NCCL halo send/recv of h_y rows",
+                       "l2_defeat": "inputs larger than L2 (a stripe is >= 512 MiB)"},
+            "tuned": {"scheme": scheme, "reach": reach, "quality_train": q_train, "tune_ms": tune_ms,
+                      "halo_y": hy, "halo_bytes_per_step_per_neighbour": hy * wd * 4},
+            "exact": {"ms_per_step": ex_ms, "value": h * wd / (ex_ms * 1e-3) / 1e6, "halo_y": r,
+                      "halo_bytes_per_step_per_neighbour": r * wd * 4},
+            "speedup_vs_exact": ex_ms / ms,
+            "roofline": {"bound": "hbm", "achieved": local_bytes / (ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                         "frac": local_bytes / (ms * 1e-3) / 1e9 / peak, "traffic": None,
+                         "kernel": approx_kernel, "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
+                         "note": "per rank: its stripe's algorithmic bytes / the max-over-ranks step time"},
+            "clocks": clk.summary(), "gpu_launches": launches,
+            "e2e": None, "cpu_baseline": None,
+        }
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -249,6 +334,8 @@ def main():
     P = pkg.paraprox
 
     dist, rank, ws, local = dist_setup()
+    if args.workload == "c4" and ws > 1:
+        return run_stripes(args, dist, rank, ws, local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()

@@ -78,8 +78,20 @@ def exchange_halos(buf: torch.Tensor, s: Stripe, hy: int, group=None, async_op: 
         raise ValueError("halo larger than the allocated capacity")
     if s.rows < hy:
         raise ValueError("stripe thinner than the halo")
-    ops = []
     c, n = s.cap, s.rows
+    if buf.is_cuda and dist.get_backend(group) == "gloo":
+        # gloo moves host tensors only: stage the halo rows through host memory
+        # (the multi-process tests on single-GPU boxes); NCCL sends device rows
+        host = buf.new_empty(buf.shape, device="cpu")
+        for r0, r1 in ((c, c + hy), (c + n - hy, c + n)):
+            host[r0:r1].copy_(buf[r0:r1])
+        exchange_halos(host, s, hy, group, async_op=False)
+        if rank > 0:
+            buf[c - hy:c].copy_(host[c - hy:c])
+        if rank < world - 1:
+            buf[c + n:c + n + hy].copy_(host[c + n:c + n + hy])
+        return []
+    ops = []
     if rank > 0:
         peer = dist.get_global_rank(group, rank - 1) if group is not None else rank - 1
         ops.append(dist.P2POp(dist.isend, buf[c:c + hy], peer, group))
