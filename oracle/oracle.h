@@ -127,6 +127,14 @@ int oracle_tune_ex(const float* x, int n, int h, int w, int separable,
                    double toq, int metric, int cap, double* qualities,
                    int* n_evaluated, int* scheme, int* rate, double* quality);
 
+/* HotSpot (Table 1; 3x3 tiles L1916-1920; NEXT-4): `iterations`
+ * explicit thermal steps T' = T + c (P + (T_N + T_S - 2T) gy + (T_E + T_W -
+ * 2T) gx + (Tamb - T) gz) on n independent [h, w] grids, the 3x3 tile of T
+ * substituted through the index maps (dy, dx) before each update. */
+int oracle_hotspot(const float* temp, const float* power, int n, int h, int w,
+                   double c, double gx, double gy, double gz, double tamb,
+                   int dy, int dx, int iterations, double* out);
+
 #ifdef __cplusplus
 }
 #endif

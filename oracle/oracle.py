@@ -74,7 +74,9 @@ def lib():
         _lib.oracle_tune_candidates_ex.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_int, i32, i32]
         _lib.oracle_tune_ex.argtypes = [f32, C.c_int, C.c_int, C.c_int, C.c_int, f32, C.c_int, f32, C.c_int,
                                         C.c_int, C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
-        for name in ("oracle_scheme_skips", "oracle_stencil_skip", "oracle_stencil_skip_sep",
+        _lib.oracle_hotspot.argtypes = [f32, f32, C.c_int, C.c_int, C.c_int, C.c_double, C.c_double, C.c_double,
+                                        C.c_double, C.c_double, C.c_int, C.c_int, C.c_int, f64]
+        for name in ("oracle_hotspot", "oracle_scheme_skips", "oracle_stencil_skip", "oracle_stencil_skip_sep",
                      "oracle_tune_candidates_ex", "oracle_tune_ex", "oracle_tune_lattice", "oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
                      "oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
                      "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
@@ -328,3 +330,18 @@ def tune_ex(x, w, toq: float, metric="mre", flags: int = 3, all_qualities: bool 
                              C.byref(q)), "tune_ex")
     return dict(scheme=SCHEME_NAMES[sc.value], reach=rc.value, quality=q.value,
                 qualities=[float(v) for v in qs[:nev.value]] if all_qualities else None)
+
+
+def hotspot(temp, power, params, dy: int = 0, dx: int = 0, iterations: int = 1) -> np.ndarray:
+    """HotSpot steps (Table 1; S25).  params = dict(c, gx, gy,
+    gz, tamb); per-axis reaches (dy, dx) substitute the 3x3 tile of T."""
+    t, squeeze = _frames(temp)
+    p, _ = _frames(power)
+    if t.shape != p.shape:
+        raise ValueError("temp and power shapes differ")
+    n, h, w = t.shape
+    out = np.empty(t.shape, dtype=np.float64)
+    _ok(lib().oracle_hotspot(_fp(t), _fp(p), n, h, w, float(params["c"]), float(params["gx"]), float(params["gy"]),
+                             float(params["gz"]), float(params["tamb"]), int(dy), int(dx), int(iterations), _dp(out)),
+        "hotspot")
+    return out[0] if squeeze else out

@@ -16,9 +16,9 @@
 namespace ppx {
 
 cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float* out, long long opitch,
-                           long long ofs, cudaStream_t s);
+                           long long ofs, cudaStream_t s, const Addend* add);
 cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, float* out, long long opitch,
-                             long long ofs, cudaStream_t s);
+                             long long ofs, cudaStream_t s, const Addend* add);
 
 void register_r1_dense();
 void register_r2_dense();
@@ -83,7 +83,7 @@ void register_tile_instance(const TileInstance& ti) {
 }
 
 static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const View& v, float* out,
-                                long long opitch, long long ofs, cudaStream_t s, bool* taken) {
+                                long long opitch, long long ofs, cudaStream_t s, const Addend* add, bool* taken) {
     *taken = false;
     int dev = 0;
     cudaError_t err = cudaGetDevice(&dev);
@@ -91,6 +91,8 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     if (dev >= kMaxDev) return cudaSuccess;
     // layout checks: TMA-describable input, 16-byte aligned output rows
     if ((reinterpret_cast<uintptr_t>(out) & 15) || (opitch & 3) || (v.n > 1 && (ofs & 3))) return cudaSuccess;
+    if (add && ((reinterpret_cast<uintptr_t>(add->p) & 15) || (add->pitch & 3) || (v.n > 1 && (add->fstride & 3))))
+        return cudaSuccess;
     const int rows_valid = v.hi - v.lo + 1;
     const long long fstride = v.n > 1 ? v.fstride : (long long)rows_valid * v.pitch;
     CUtensorMap tmap;
@@ -127,6 +129,11 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.out = out;
     A.opitch = opitch;
     A.ofs = ofs;
+    A.addp = add ? add->p : nullptr;
+    A.apitch = add ? add->pitch : 0;
+    A.afs = add ? add->fstride : 0;
+    A.alpha = add ? add->alpha : 0.f;
+    A.beta = add ? add->beta : 0.f;
     TapW W = {};
     if (p.separable) {
         for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 8] = p.wyf[i];
@@ -155,21 +162,21 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
 }
 
 cudaError_t launch_stencil(const Plan& p, const float* in, const View& v, float* out, long long opitch,
-                           long long ofs, cudaStream_t s) {
+                           long long ofs, cudaStream_t s, const Addend* add) {
     // a plan that accesses only the centre is a map: stream it (k_pointwise.cu)
-    if (!force_generic() && p.hy == 0 && p.hx == 0) return launch_pointwise(p, in, v, out, opitch, ofs, s);
+    if (!force_generic() && p.hy == 0 && p.hx == 0) return launch_pointwise(p, in, v, out, opitch, ofs, s, add);
     const int rmax = p.separable ? 8 : 4;  // tile instances: dense r <= 4, separable r <= 8
     if (!force_generic() && p.ry <= rmax && p.rx <= rmax) {
         init_registry();
         for (Entry& e : reg()) {
             if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;
             bool taken = false;
-            cudaError_t err = launch_tiles(e, p, in, v, out, opitch, ofs, s, &taken);
+            cudaError_t err = launch_tiles(e, p, in, v, out, opitch, ofs, s, add, &taken);
             if (err != cudaSuccess || taken) return err;
             break;
         }
     }
-    return launch_generic(p, in, v, out, opitch, ofs, s);
+    return launch_generic(p, in, v, out, opitch, ofs, s, add);
 }
 
 }  // namespace ppx

@@ -79,11 +79,19 @@ struct View {
     int lo, hi;  // valid input rows: [lo, hi] relative to row 0 (lo = -halo_top)
 };
 
+// An additive second input (HotSpot's power term, NEXT-4):
+// out = stencil(in) + alpha * p[f, y, x] + beta, p laid out like the output.
+struct Addend {
+    const float* p = nullptr;
+    long long pitch = 0, fstride = 0;
+    float alpha = 0.f, beta = 0.f;
+};
+
 // ---- kernels ----
 // Each launcher enqueues on `s`, bumps the launch counter, records the kernel
 // name and returns cudaGetLastError().
 cudaError_t launch_stencil(const Plan& p, const float* in, const View& vin, float* out,
-                           long long out_pitch, long long out_fstride, cudaStream_t s);
+                           long long out_pitch, long long out_fstride, cudaStream_t s, const Addend* add = nullptr);
 // global-lattice stencil (k_lattice.cu): exact stencil on the array rebuilt
 // from the accessed rows/columns (reaches dy, dx); halos must be 0
 cudaError_t launch_lattice(const paraprox_filter_s& f, const float* in, const View& v, float* out,

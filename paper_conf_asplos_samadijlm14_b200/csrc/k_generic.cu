@@ -15,7 +15,8 @@ struct TapTable {
 
 __global__ void __launch_bounds__(256) k_stencil_generic(const float* __restrict__ in, View v,
                                                          float* __restrict__ out, long long opitch,
-                                                         long long ofs, const __grid_constant__ TapTable t) {
+                                                         long long ofs, const __grid_constant__ TapTable t,
+                                                         const Addend add) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
     const int y = blockIdx.y * blockDim.y + threadIdx.y;
     if (x >= v.w || y >= v.h) return;
@@ -27,6 +28,9 @@ __global__ void __launch_bounds__(256) k_stencil_generic(const float* __restrict
             const int xx = min(max(x + (int)t.ox[k], 0), v.w - 1);
             acc = fmaf(t.w[k], __ldg(F + (long long)yy * v.pitch + xx), acc);
         }
+        if (add.p)
+            acc = __fadd_rn(__fmaf_rn(add.alpha, add.p[(long long)f * add.fstride + (long long)y * add.pitch + x], acc),
+                            add.beta);
         out[(long long)f * ofs + (long long)y * opitch + x] = acc;
     }
 }
@@ -45,12 +49,12 @@ static void fill_taps(const Plan& p, TapTable* t) {
 }
 
 cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float* out, long long opitch,
-                           long long ofs, cudaStream_t s) {
+                           long long ofs, cudaStream_t s, const Addend* add) {
     TapTable t;
     fill_taps(p, &t);
     dim3 block(32, 8);
     dim3 grid((v.w + 31) / 32, (v.h + 7) / 8, v.n < 65535 ? v.n : 65535);
-    k_stencil_generic<<<grid, block, 0, s>>>(in, v, out, opitch, ofs, t);
+    k_stencil_generic<<<grid, block, 0, s>>>(in, v, out, opitch, ofs, t, add ? *add : Addend());
     count_launch("generic");
     return cudaGetLastError();
 }

@@ -27,10 +27,17 @@ __device__ __forceinline__ float4 pw4(float4 x, float w0, float w1) {
     return make_float4(pw<SEP>(x.x, w0, w1), pw<SEP>(x.y, w0, w1), pw<SEP>(x.z, w0, w1), pw<SEP>(x.w, w0, w1));
 }
 
+__device__ __forceinline__ float plus(float r, float a, const Addend& add) {
+    return __fadd_rn(__fmaf_rn(add.alpha, a, r), add.beta);
+}
+__device__ __forceinline__ float4 plus4(float4 r, float4 a, const Addend& add) {
+    return make_float4(plus(r.x, a.x, add), plus(r.y, a.y, add), plus(r.z, a.z, add), plus(r.w, a.w, add));
+}
+
 // contiguous input and output, 16-byte aligned: one flat array
 template <bool SEP>
 __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict__ in, float* __restrict__ out,
-                                                        long long count, float w0, float w1) {
+                                                        long long count, float w0, float w1, const Addend add) {
     const long long n4 = count >> 2;
     const long long stride = (long long)gridDim.x * blockDim.x;
     const float4* i4 = reinterpret_cast<const float4*>(in);
@@ -44,17 +51,22 @@ __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict_
             if (i + u * stride < n4) v[u] = __ldcs(i4 + i + u * stride);
 #pragma unroll
         for (int u = 0; u < kPU; ++u)
-            if (i + u * stride < n4) __stcs(o4 + i + u * stride, pw4<SEP>(v[u], w0, w1));
+            if (i + u * stride < n4) {
+                float4 r = pw4<SEP>(v[u], w0, w1);
+                if (add.p) r = plus4(r, __ldcs(reinterpret_cast<const float4*>(add.p) + i + u * stride), add);
+                __stcs(o4 + i + u * stride, r);
+            }
     }
     if (blockIdx.x == 0)
-        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) out[x] = pw<SEP>(in[x], w0, w1);
+        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x)
+            out[x] = add.p ? plus(pw<SEP>(in[x], w0, w1), add.p[x], add) : pw<SEP>(in[x], w0, w1);
 }
 
 // any layout: rows of the output image, 128-bit where both rows allow it
 template <bool SEP>
 __global__ void __launch_bounds__(256) k_pointwise_rows(const float* __restrict__ in, View v,
                                                         float* __restrict__ out, long long opitch,
-                                                        long long ofs, float w0, float w1) {
+                                                        long long ofs, float w0, float w1, const Addend add) {
     const long long rows = (long long)v.n * v.h;
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -62,16 +74,26 @@ __global__ void __launch_bounds__(256) k_pointwise_rows(const float* __restrict_
         const long long f = R / v.h, y = R - f * v.h;
         const float* src = in + f * v.fstride + y * v.pitch;
         float* dst = out + f * ofs + y * opitch;
-        const bool vec = ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15) == 0;
+        const float* ap = add.p ? add.p + f * add.fstride + y * add.pitch : nullptr;
+        const bool vec = ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst) |
+                           reinterpret_cast<uintptr_t>(ap)) & 15) == 0;
         const int w4 = vec ? (v.w >> 2) : 0;
-        for (int x = threadIdx.x; x < w4; x += blockDim.x)
-            __stcs(reinterpret_cast<float4*>(dst) + x, pw4<SEP>(__ldcs(reinterpret_cast<const float4*>(src) + x), w0, w1));
-        for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x) __stcs(dst + x, pw<SEP>(__ldcs(src + x), w0, w1));
+        for (int x = threadIdx.x; x < w4; x += blockDim.x) {
+            float4 r = pw4<SEP>(__ldcs(reinterpret_cast<const float4*>(src) + x), w0, w1);
+            if (ap) r = plus4(r, __ldcs(reinterpret_cast<const float4*>(ap) + x), add);
+            __stcs(reinterpret_cast<float4*>(dst) + x, r);
+        }
+        for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x) {
+            float r = pw<SEP>(__ldcs(src + x), w0, w1);
+            if (ap) r = plus(r, __ldcs(ap + x), add);
+            __stcs(dst + x, r);
+        }
     }
 }
 
 cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, float* out, long long opitch,
-                             long long ofs, cudaStream_t s) {
+                             long long ofs, cudaStream_t s, const Addend* addp) {
+    const Addend add = addp ? *addp : Addend();
     static int sms[64] = {};
     int dev = 0;
     cudaError_t err = cudaGetDevice(&dev);
@@ -87,7 +109,9 @@ cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, floa
     const long long count = (long long)v.n * v.h * v.w;
     const bool flat = v.pitch == v.w && opitch == v.w && (v.n == 1 || (v.fstride == (long long)v.h * v.w &&
                       ofs == (long long)v.h * v.w)) &&
-                      (((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15) == 0);
+                      (((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15) == 0) &&
+                      (!add.p || (add.pitch == v.w && (v.n == 1 || add.fstride == (long long)v.h * v.w) &&
+                                  (reinterpret_cast<uintptr_t>(add.p) & 15) == 0));
     cudaLaunchConfig_t cfg = {};
     cfg.blockDim = dim3(256);
     cfg.stream = s;
@@ -100,14 +124,14 @@ cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, floa
     if (flat) {
         const long long want = (count / 4 + 255) / 256;
         cfg.gridDim = dim3((unsigned)(want < resident ? (want > 0 ? want : 1) : resident));
-        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_flat<true>, in, out, count, w0, w1)
-                          : cudaLaunchKernelEx(&cfg, k_pointwise_flat<false>, in, out, count, w0, w1);
+        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_flat<true>, in, out, count, w0, w1, add)
+                          : cudaLaunchKernelEx(&cfg, k_pointwise_flat<false>, in, out, count, w0, w1, add);
         count_launch(p.separable ? "sep_map" : "dense_map");
     } else {
         const long long rows = (long long)v.n * v.h;
         cfg.gridDim = dim3((unsigned)(rows < resident ? rows : resident));
-        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_rows<true>, in, v, out, opitch, ofs, w0, w1)
-                          : cudaLaunchKernelEx(&cfg, k_pointwise_rows<false>, in, v, out, opitch, ofs, w0, w1);
+        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_rows<true>, in, v, out, opitch, ofs, w0, w1, add)
+                          : cudaLaunchKernelEx(&cfg, k_pointwise_rows<false>, in, v, out, opitch, ofs, w0, w1, add);
         count_launch(p.separable ? "sep_map_rows" : "dense_map_rows");
     }
     if (err != cudaSuccess) return err;

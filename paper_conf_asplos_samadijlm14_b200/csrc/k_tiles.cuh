@@ -52,6 +52,9 @@ struct TileArgs {
     int tiles_x, tiles_y, ntiles;
     float* out;
     long long opitch, ofs;
+    const float* addp;  // optional additive input (NEXT-4): out += alpha * addp + beta
+    long long apitch, afs;
+    float alpha, beta;
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -272,15 +275,29 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         // stores: 128-bit streaming where the 4 columns are inside the image
         const int x = x0 + 4 * lane;
         float* obase = A.out + (long long)f * A.ofs + x;
+        const float* abase = A.addp ? A.addp + (long long)f * A.afs + x : nullptr;
 #pragma unroll
         for (int k = 0; k < kRB; ++k) {
             const int y = y0 + ty0 + k;
             if (y < A.h && x < A.w) {
                 float* o = obase + (long long)y * A.opitch;
+                float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
+                if (abase) {
+                    const float* ap = abase + (long long)y * A.apitch;
+                    float a4[4];
+                    if (x + 3 < A.w) {
+                        const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
+                        a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) a4[c] = x + c < A.w ? ap[c] : 0.f;
+                    }
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
+                }
                 if (x + 3 < A.w) {
-                    __stcs(reinterpret_cast<float4*>(o), make_float4(acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y));
+                    __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
                 } else {
-                    const float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
 #pragma unroll
                     for (int c = 0; c < 4; ++c)
                         if (x + c < A.w) __stcs(o + c, r4[c]);
