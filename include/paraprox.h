@@ -173,6 +173,25 @@ PARAPROX_API paraprox_status paraprox_run_host(paraprox_filter f, paraprox_schem
                                   const float* h_in, float* h_out, const paraprox_image* img,
                                   paraprox_stream s);
 
+/* ---- HotSpot: an iterated Stencil-Partition application (NEXT-4) -------- */
+
+/* HotSpot (Table 1: 1024x1024, Stencil-Partition, MRE; 3x3 tiles,
+ * L1916-1920).  `iterations` explicit thermal steps of the Rodinia kernel
+ * (reading S25):
+ *   T'(y,x) = T + c (P + (T_N + T_S - 2T) gy + (T_E + T_W - 2T) gx + (Tamb - T) gz)
+ * with c = step_div_cap, gx = rx_inv, gy = ry_inv, gz = rz_inv; the 3x3 tile of
+ * T read by each step is approximated by (scheme, reach) like a stencil (row:
+ * the north/south reads take the centre row, ...).  d_temp, d_power and d_out
+ * share img's layout (n independent grids); d_temp is not modified; halos are
+ * allowed only with iterations == 1 (one step of a row stripe).  Scratch: one
+ * image, stream-ordered.  Asynchronous on s. */
+typedef struct {
+    double step_div_cap, rx_inv, ry_inv, rz_inv, t_amb;
+} paraprox_hotspot_params;
+PARAPROX_API paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_scheme scheme,
+                                 int reach, const float* d_temp, const float* d_power, float* d_out,
+                                 const paraprox_image* img, int iterations, paraprox_stream s);
+
 /* ---- output quality (syncs s) ------------------------------------------ */
 
 /* Quality of d_approx against d_exact over all n*h*w elements (pooled over

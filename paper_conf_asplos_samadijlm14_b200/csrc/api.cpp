@@ -440,6 +440,61 @@ paraprox_status paraprox_tune_lattice(paraprox_filter f, const float* d_train, c
     return paraprox_tune_lattice_decide(parts, m, toq, out_scheme, out_reach, out_quality);
 }
 
+paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_scheme scheme, int reach,
+                                 const float* d_temp, const float* d_power, float* d_out, const paraprox_image* img,
+                                 int iterations, paraprox_stream s) {
+    if (!prm || !d_temp || !d_power || !d_out) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0) return fail(PARAPROX_ERR_INVALID_ARG, "reach < 0");
+    if (iterations < 1) return fail(PARAPROX_ERR_INVALID_ARG, "iterations < 1");
+    paraprox_status st = check_image(img, iterations == 1);
+    if (st != PARAPROX_OK) return st;
+    if (overlaps(d_temp, d_out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_temp");
+    paraprox_image pimg = *img;  // the power grid has the output's rows only
+    pimg.halo_top = pimg.halo_bottom = 0;
+    if (overlaps(d_power, d_out, &pimg)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_power");
+    // the step as a 3x3 filter on T plus an additive power term (reading S25):
+    // T' = sum w T + c P + c gz Tamb, w = [[0, c gy, 0], [c gx, 1 - 2c gx - 2c gy - c gz, c gx], [0, c gy, 0]]
+    const double c = prm->step_div_cap, gx = prm->rx_inv, gy = prm->ry_inv, gz = prm->rz_inv;
+    paraprox_filter_s f;
+    f.ky = f.kx = 3;
+    f.separable = false;
+    f.w = {0.f, (float)(c * gy), 0.f, (float)(c * gx), (float)(1.0 - 2.0 * c * gx - 2.0 * c * gy - c * gz),
+           (float)(c * gx), 0.f, (float)(c * gy), 0.f};
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    const Plan& p = get_plan(&f, dy, dx);
+    cudaStream_t cs = (cudaStream_t)s;
+    const View v0 = view_of(img);
+    const long long ofs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
+    Addend add;
+    add.p = d_power;
+    add.pitch = img->pitch;
+    add.fstride = ofs;
+    add.alpha = (float)c;
+    add.beta = (float)(c * gz * prm->t_amb);
+    // ping-pong between d_out and one scratch image so that the last step
+    // lands in d_out; d_temp is never written
+    DevBuf buf;
+    buf.s = cs;
+    if (iterations > 1) {
+        const size_t need = (size_t)((img->n - 1) * ofs + (long long)(img->h - 1) * img->pitch + img->w);
+        PPX_CUDA(scratch_alloc(&buf.p, need * sizeof(float), cs));
+    }
+    View vn = v0;  // later steps read an image with the output's layout, no halos
+    vn.fstride = ofs;
+    vn.lo = 0;
+    vn.hi = img->h - 1;
+    const float* src = d_temp;
+    for (int it = 0; it < iterations; ++it) {
+        float* dst = ((iterations - 1 - it) % 2 == 0) ? d_out : (float*)buf.p;
+        cudaError_t e = launch_stencil(p, src, it == 0 ? v0 : vn, dst, img->pitch, ofs, cs, &add);
+        if (e != cudaSuccess) return cuda_fail(e, "hotspot step");
+        src = dst;
+    }
+    return PARAPROX_OK;
+}
+
 paraprox_status paraprox_quality(const float* d_exact, const float* d_approx, const paraprox_image* img,
                                  paraprox_metric m, double* h_quality, paraprox_stream s) {
     if (!h_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");

@@ -35,6 +35,11 @@ METRICS = {"mre": MRE, "l2": L2, "psnr": PSNR}
 MAX_K = 17
 
 
+class HotspotParams(C.Structure):
+    _fields_ = [("step_div_cap", C.c_double), ("rx_inv", C.c_double), ("ry_inv", C.c_double),
+                ("rz_inv", C.c_double), ("t_amb", C.c_double)]
+
+
 class Image(C.Structure):
     _fields_ = [("n", C.c_int), ("h", C.c_int), ("w", C.c_int), ("pitch", C.c_longlong),
                 ("frame_stride", C.c_longlong), ("halo_top", C.c_int), ("halo_bottom", C.c_int)]
@@ -56,6 +61,7 @@ _SIGS = {
     "paraprox_run_host": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_stencil_lattice": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_stencil_skip_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
+    "paraprox_hotspot": [C.POINTER(HotspotParams), C.c_int, C.c_int, _P, _P, _P, _IMG, C.c_int, _P],
     "paraprox_tune_ex": [_P, C.c_int, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
     "paraprox_tune_candidates_ex": [_P, C.c_int, C.c_int, _I, _I, _I],
     "paraprox_tune_partials_ex": [_P, C.c_int, _P, _IMG, C.c_int, _D, _P],
@@ -574,3 +580,19 @@ def tune_decide_ex(f: Filter, partials, toq: float, metric="mre", flags: int = 3
                                         _metric(metric), float(toq), C.byref(sc), C.byref(rc), C.byref(q)),
            "tune_decide_ex")
     return SCHEME_NAMES[sc.value], rc.value, q.value
+
+
+def hotspot(temp, power, params, scheme="exact", reach: int = 0, iterations: int = 1, out=None, *, halo_top=0,
+            halo_bottom=0, stream=None):
+    """HotSpot steps (paraprox_hotspot).  params: dict(c, gx, gy, gz, tamb)."""
+    _need_cuda(temp, power)
+    img = image_of(temp, halo_top, halo_bottom)
+    out = _out_like(temp, halo_top, halo_bottom, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check_out(power, img)
+    prm = HotspotParams(float(params["c"]), float(params["gx"]), float(params["gy"]), float(params["gz"]),
+                        float(params["tamb"]))
+    _check(_lib.paraprox_hotspot(C.byref(prm), _scheme(scheme), int(reach), _dp(temp, halo_top), _dp(power), _dp(out),
+                                 C.byref(img), int(iterations), _stream(stream)), "hotspot")
+    return out

@@ -1,0 +1,92 @@
+"""GPU parity of the HotSpot steps (NEXT-4; Table 1, 3x3 tiles
+L1916-1920; reading S25) against the oracle: every scheme, several iteration
+counts, the paper's 1024x1024 size, a row stripe, a misaligned layout.
+
+Tolerance: the GPU keeps fp32 state, the oracle fp64; per output
+|gpu - oracle| <= 1e-5 * |oracle| (temperatures are ~330 K)."""
+import numpy as np
+import pytest
+import torch
+
+from workloads import hotspot as H
+
+pytestmark = pytest.mark.gpu
+
+PRM = H.PARAMS
+
+
+@pytest.fixture(scope="module")
+def P():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_asplos_samadijlm14_b200 as pkg
+
+    return pkg.paraprox
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+SCHEMES = [("exact", 0, (0, 0)), ("row", 1, (1, 0)), ("col", 1, (0, 1)), ("center", 1, (1, 1))]
+
+
+@pytest.mark.parametrize("scheme,reach,dd", SCHEMES, ids=[s[0] for s in SCHEMES])
+@pytest.mark.parametrize("iters", [1, 2, 7])
+def test_parity(P, O, scheme, reach, dd, iters):
+    t, p = H.frames(2, 96, 160, 1)
+    g = P.hotspot(dev(t), dev(p), PRM, scheme, reach, iters).cpu().numpy()
+    o = O.hotspot(t, p, PRM, dd[0], dd[1], iters)
+    assert np.all(np.abs(g - o) <= 1e-5 * np.abs(o)), (scheme, iters, float(np.abs(g - o).max()))
+
+
+@pytest.mark.parametrize("scheme,reach,dd", SCHEMES, ids=[s[0] for s in SCHEMES])
+def test_paper_size_1024(P, O, scheme, reach, dd):
+    t, p = H.frames(1, 1024, 1024, 5)
+    g = P.hotspot(dev(t), dev(p), PRM, scheme, reach, 20).cpu().numpy()
+    o = O.hotspot(t, p, PRM, dd[0], dd[1], 20)
+    assert np.all(np.abs(g - o) <= 1e-5 * np.abs(o)), (scheme, float(np.abs(g - o).max()))
+    k = P.last_kernel()
+    assert k == ("dense_map" if scheme == "center" else k) and k != "generic", k
+
+
+def test_reach_saturates_and_input_untouched(P):
+    t, p = H.frames(1, 64, 64, 2)
+    td = dev(t)
+    a = P.hotspot(td, dev(p), PRM, "row", 1, 3)
+    b = P.hotspot(td, dev(p), PRM, "row", 5, 3)
+    assert torch.equal(a, b)
+    assert torch.equal(td, dev(t))
+
+
+def test_stripe_step_equals_whole_grid(P):
+    t, p = H.frames(1, 120, 256, 3)
+    full = P.hotspot(dev(t[0]), dev(p[0]), PRM, "exact", 0, 1)
+    r0, r1 = 40, 80
+    stripe_t = dev(t[0][r0 - 1:r1 + 1])
+    got = P.hotspot(stripe_t, dev(p[0][r0:r1]), PRM, "exact", 0, 1, halo_top=1, halo_bottom=1,
+                    out=torch.empty(r1 - r0 + 2, 256, device="cuda")[1:-1])
+    assert torch.equal(got, full[r0:r1])
+
+
+def test_misaligned_layout_generic(P, O):
+    t, p = H.frames(1, 50, 77, 4)
+    n = 50 * 77
+    bt, bp, bo = (torch.zeros(n + 1, device="cuda") for _ in range(3))
+    tv, pv, ov = bt[1:].view(50, 77), bp[1:].view(50, 77), bo[1:].view(50, 77)
+    tv.copy_(dev(t[0]))
+    pv.copy_(dev(p[0]))
+    g = P.hotspot(tv, pv, PRM, "exact", 0, 4, out=ov).cpu().numpy()
+    o = O.hotspot(t[0], p[0], PRM, 0, 0, 4)
+    assert np.all(np.abs(g - o) <= 1e-5 * np.abs(o))
+    assert P.last_kernel() == "generic"
+
+
+def test_quality_of_the_approximation(P):
+    """MRE of each scheme after 20 steps of the 1024^2 grid (reported)."""
+    t, p = H.frames(1, 1024, 1024, 6)
+    e = P.hotspot(dev(t), dev(p), PRM, "exact", 0, 20)
+    for scheme in ("row", "col", "center"):
+        a = P.hotspot(dev(t), dev(p), PRM, scheme, 1, 20)
+        q = P.quality(e, a, "mre")
+        print(f"hotspot 1024^2 x20 {scheme}: quality {q:.6f}")
+        assert 0.9 < q < 1.0
