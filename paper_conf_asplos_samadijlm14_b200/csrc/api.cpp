@@ -486,6 +486,14 @@ paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_sc
     vn.lo = 0;
     vn.hi = img->h - 1;
     const float* src = d_temp;
+    if (p.hy == 0 && p.hx == 0) {
+        // the centre scheme at full reach reads no neighbour: all the steps
+        // fuse into one pass (k_pointwise), one HBM round trip for `iterations`
+        add.steps = iterations;
+        cudaError_t e = launch_stencil(p, src, v0, d_out, img->pitch, ofs, cs, &add);
+        if (e != cudaSuccess) return cuda_fail(e, "hotspot fused steps");
+        return PARAPROX_OK;
+    }
     for (int it = 0; it < iterations; ++it) {
         float* dst = ((iterations - 1 - it) % 2 == 0) ? d_out : (float*)buf.p;
         cudaError_t e = launch_stencil(p, src, it == 0 ? v0 : vn, dst, img->pitch, ofs, cs, &add);

@@ -85,6 +85,7 @@ struct Addend {
     const float* p = nullptr;
     long long pitch = 0, fstride = 0;
     float alpha = 0.f, beta = 0.f;
+    int steps = 1;  // centre-only plans (k_pointwise): x <- w' x + alpha p + beta, `steps` times
 };
 
 // ---- kernels ----

@@ -28,9 +28,13 @@ __global__ void __launch_bounds__(256) k_stencil_generic(const float* __restrict
             const int xx = min(max(x + (int)t.ox[k], 0), v.w - 1);
             acc = fmaf(t.w[k], __ldg(F + (long long)yy * v.pitch + xx), acc);
         }
-        if (add.p)
-            acc = __fadd_rn(__fmaf_rn(add.alpha, add.p[(long long)f * add.fstride + (long long)y * add.pitch + x], acc),
-                            add.beta);
+        if (add.p) {
+            const float a = add.p[(long long)f * add.fstride + (long long)y * add.pitch + x];
+            acc = __fadd_rn(__fmaf_rn(add.alpha, a, acc), add.beta);
+            // fused steps of a centre-only plan (one tap at (0, 0)), as k_pointwise
+            for (int k = 1; k < add.steps; ++k)
+                acc = __fadd_rn(__fmaf_rn(add.alpha, a, __fmaf_rn(t.w[0], acc, 0.f)), add.beta);
+        }
         out[(long long)f * ofs + (long long)y * opitch + x] = acc;
     }
 }

@@ -33,6 +33,19 @@ __device__ __forceinline__ float plus(float r, float a, const Addend& add) {
 __device__ __forceinline__ float4 plus4(float4 r, float4 a, const Addend& add) {
     return make_float4(plus(r.x, a.x, add), plus(r.y, a.y, add), plus(r.z, a.z, add), plus(r.w, a.w, add));
 }
+// a centre-only plan has no neighbours, so consecutive steps of an iterated
+// map (HotSpot at full collapse) fuse: the value stays in a register, each
+// step rounded exactly as a separate launch would round it
+template <bool SEP>
+__device__ __forceinline__ float4 steps4(float4 x, float4 a, float w0, float w1, const Addend& add) {
+    for (int k = 0; k < add.steps; ++k) x = plus4(pw4<SEP>(x, w0, w1), a, add);
+    return x;
+}
+template <bool SEP>
+__device__ __forceinline__ float steps1(float x, float a, float w0, float w1, const Addend& add) {
+    for (int k = 0; k < add.steps; ++k) x = plus(pw<SEP>(x, w0, w1), a, add);
+    return x;
+}
 
 // contiguous input and output, 16-byte aligned: one flat array
 template <bool SEP>
@@ -52,14 +65,15 @@ __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict_
 #pragma unroll
         for (int u = 0; u < kPU; ++u)
             if (i + u * stride < n4) {
-                float4 r = pw4<SEP>(v[u], w0, w1);
-                if (add.p) r = plus4(r, __ldcs(reinterpret_cast<const float4*>(add.p) + i + u * stride), add);
+                float4 r = add.p ? steps4<SEP>(v[u], __ldcs(reinterpret_cast<const float4*>(add.p) + i + u * stride),
+                                               w0, w1, add)
+                                 : pw4<SEP>(v[u], w0, w1);
                 __stcs(o4 + i + u * stride, r);
             }
     }
     if (blockIdx.x == 0)
         for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x)
-            out[x] = add.p ? plus(pw<SEP>(in[x], w0, w1), add.p[x], add) : pw<SEP>(in[x], w0, w1);
+            out[x] = add.p ? steps1<SEP>(in[x], add.p[x], w0, w1, add) : pw<SEP>(in[x], w0, w1);
 }
 
 // any layout: rows of the output image, 128-bit where both rows allow it
@@ -79,13 +93,13 @@ __global__ void __launch_bounds__(256) k_pointwise_rows(const float* __restrict_
                            reinterpret_cast<uintptr_t>(ap)) & 15) == 0;
         const int w4 = vec ? (v.w >> 2) : 0;
         for (int x = threadIdx.x; x < w4; x += blockDim.x) {
-            float4 r = pw4<SEP>(__ldcs(reinterpret_cast<const float4*>(src) + x), w0, w1);
-            if (ap) r = plus4(r, __ldcs(reinterpret_cast<const float4*>(ap) + x), add);
+            const float4 xv = __ldcs(reinterpret_cast<const float4*>(src) + x);
+            const float4 r = ap ? steps4<SEP>(xv, __ldcs(reinterpret_cast<const float4*>(ap) + x), w0, w1, add)
+                                : pw4<SEP>(xv, w0, w1);
             __stcs(reinterpret_cast<float4*>(dst) + x, r);
         }
         for (int x = (w4 << 2) + threadIdx.x; x < v.w; x += blockDim.x) {
-            float r = pw<SEP>(__ldcs(src + x), w0, w1);
-            if (ap) r = plus(r, __ldcs(ap + x), add);
+            const float r = ap ? steps1<SEP>(__ldcs(src + x), __ldcs(ap + x), w0, w1, add) : pw<SEP>(__ldcs(src + x), w0, w1);
             __stcs(dst + x, r);
         }
     }

@@ -198,6 +198,28 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         }
 
         const int ty0 = wi * kRB;
+        // the additive input (HotSpot's power) is loaded before the compute so
+        // its latency hides behind the FMAs
+        const int xo = x0 + 4 * lane;
+        float4 pv[kRB];
+        if (A.addp) {
+            const float* abase = A.addp + (long long)f * A.afs + xo;
+#pragma unroll
+            for (int k = 0; k < kRB; ++k) {
+                const int y = y0 + ty0 + k;
+                pv[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (y < A.h && xo < A.w) {
+                    const float* ap = abase + (long long)y * A.apitch;
+                    if (xo + 3 < A.w) {
+                        pv[k] = __ldcs(reinterpret_cast<const float4*>(ap));
+                    } else {
+                        pv[k].x = ap[0];
+                        if (xo + 1 < A.w) pv[k].y = ap[1];
+                        if (xo + 2 < A.w) pv[k].z = ap[2];
+                    }
+                }
+            }
+        }
         // outputs as column pairs (c = 0,1 and 2,3): every FMA is a packed
         // FFMA2 (fma.rn.f32x2, sm_100) -- the same fp32 fma per lane, so the
         // per-pixel rounding and tap order are unchanged, at half the issue
@@ -275,23 +297,14 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         // stores: 128-bit streaming where the 4 columns are inside the image
         const int x = x0 + 4 * lane;
         float* obase = A.out + (long long)f * A.ofs + x;
-        const float* abase = A.addp ? A.addp + (long long)f * A.afs + x : nullptr;
 #pragma unroll
         for (int k = 0; k < kRB; ++k) {
             const int y = y0 + ty0 + k;
             if (y < A.h && x < A.w) {
                 float* o = obase + (long long)y * A.opitch;
                 float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
-                if (abase) {
-                    const float* ap = abase + (long long)y * A.apitch;
-                    float a4[4];
-                    if (x + 3 < A.w) {
-                        const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
-                        a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
-                    } else {
-#pragma unroll
-                        for (int c = 0; c < 4; ++c) a4[c] = x + c < A.w ? ap[c] : 0.f;
-                    }
+                if (A.addp) {
+                    const float a4[4] = {pv[k].x, pv[k].y, pv[k].z, pv[k].w};
 #pragma unroll
                     for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
                 }

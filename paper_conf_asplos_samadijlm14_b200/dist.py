@@ -150,6 +150,46 @@ def stencil_stripe(buf: torch.Tensor, s: Stripe, f, scheme, reach: int, out: tor
     return out
 
 
+def hotspot_stripes(bufs, power: torch.Tensor, s: Stripe, params, scheme, reach: int, iterations: int,
+                    group=None, compute=None):
+    """`iterations` HotSpot steps (NEXT-4) of a row-striped grid: before each
+    step the stripe exchanges the h_y halo rows of the current temperature
+    with its neighbours (exact and column schemes read the north/south
+    neighbours: h_y = 1; the row and centre schemes at reach >= 1 read only
+    the centre row: h_y = 0, no exchange at all), overlapped with the interior
+    rows; then the boundary rows.  `bufs` = two [cap + rows + cap, w] buffers,
+    the initial temperature in bufs[0]'s owned rows; `power` = [rows, w].
+    Returns the buffer holding the final owned rows.  `compute(band, ht, hb,
+    power_rows, out_rows)` defaults to one paraprox_hotspot step."""
+    if compute is None:
+        from . import paraprox as P
+
+        def compute(band, ht, hb, pw, o):
+            P.hotspot(band, pw, params, scheme, reach, 1, out=o, halo_top=ht, halo_bottom=hb)
+    hy = 1 if (scheme == "exact" or reach == 0 or scheme in ("col", "column")) else 0
+    n, c = s.rows, s.cap
+    ht, hb = s.halo_top(hy), s.halo_bottom(hy)
+    cur, nxt = bufs
+    for _ in range(iterations):
+        out = nxt[c:c + n]
+        if hy == 0 or n <= 2 * hy:
+            exchange_halos(cur, s, hy, group)
+            band, t, b = _band(cur, s, 0, n, ht, hb)
+            compute(band, t, b, power, out)
+        else:
+            reqs = exchange_halos(cur, s, hy, group, async_op=True)
+            band, t, b = _band(cur, s, hy, n - hy, hy, hy)
+            compute(band, t, b, power[hy:n - hy], out[hy:n - hy])
+            for r in reqs:
+                r.wait()
+            band, t, b = _band(cur, s, 0, hy, ht, min(hy, n - hy))
+            compute(band, t, b, power[0:hy], out[0:hy])
+            band, t, b = _band(cur, s, n - hy, n, min(hy, n - hy), hb)
+            compute(band, t, b, power[n - hy:n], out[n - hy:n])
+        cur, nxt = nxt, cur
+    return cur
+
+
 def _allreduce_np(a: np.ndarray, device, group=None) -> np.ndarray:
     t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).to(device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)

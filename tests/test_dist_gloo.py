@@ -73,6 +73,46 @@ def _worker_stripes(rank, world, port, q):
             dist.destroy_process_group()
 
 
+def _worker_hotspot(rank, world, port, q):
+    try:
+        _init(rank, world, port)
+        import oracle as O
+        from paper_conf_asplos_samadijlm14_b200 import dist as D
+        from workloads import hotspot as H
+        h, w, iters = 37, 23, 5
+        t, p = H.frames(1, h, w, 4)
+        t, p = t[0], p[0]
+        prm = H.PARAMS
+        s = D.stripe_of(h, world, rank, cap=1)
+        for scheme, reach, dd in (("exact", 0, (0, 0)), ("row", 1, (1, 0)), ("col", 1, (0, 1)),
+                                  ("center", 1, (1, 1))):
+            full = O.hotspot(t, p, prm, dd[0], dd[1], iters)
+            bufs = [D.alloc_stripe(s, w, dtype=torch.float64) for _ in range(2)]
+            for b in bufs:
+                b.fill_(float("nan"))
+            bufs[0][s.cap:s.cap + s.rows] = torch.from_numpy(t[s.r0:s.r1].astype(np.float64))
+            pw = torch.from_numpy(p[s.r0:s.r1].astype(np.float64))
+
+            def compute(band, ht, hb, pwr, o):
+                bnd = band.numpy()
+                assert not np.isnan(bnd).any(), "read an unexchanged halo row"
+                res = O.hotspot(bnd.astype(np.float32), np.pad(pwr.numpy(), ((ht, hb), (0, 0))).astype(np.float32),
+                                prm, dd[0], dd[1], 1)
+                o.copy_(torch.from_numpy(res[ht:ht + o.shape[0]]))
+
+            fin = D.hotspot_stripes(bufs, pw, s, prm, scheme, reach, iters, compute=compute)
+            got = fin[s.cap:s.cap + s.rows].numpy()
+            # the oracle band steps round the state to fp32 between steps: compare at fp32 precision
+            assert np.allclose(got, full[s.r0:s.r1], rtol=1e-6, atol=0), (rank, scheme)
+        q.put((rank, "ok"))
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, traceback.format_exc()))
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
 def _worker_exchange(rank, world, port, q):
     try:
         _init(rank, world, port)
@@ -174,3 +214,8 @@ def test_frame_shard_covers():
             assert got[0][0] == 0 and got[-1][1] == n
             assert all(got[i][1] == got[i + 1][0] for i in range(world - 1))
             assert max(b - a for a, b in got) - min(b - a for a, b in got) <= 1
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_hotspot_stripes_reproduce_whole_grid(world):
+    _run(_worker_hotspot, world)

@@ -90,3 +90,15 @@ def test_quality_of_the_approximation(P):
         q = P.quality(e, a, "mre")
         print(f"hotspot 1024^2 x20 {scheme}: quality {q:.6f}")
         assert 0.9 < q < 1.0
+
+
+def test_fused_centre_steps_equal_single_steps(P):
+    """Full collapse reads no neighbour, so the steps fuse into one pass; the
+    result is bit-identical to one launch per step."""
+    t, p = H.frames(2, 64, 96, 7)
+    td, pd = dev(t), dev(p)
+    fused = P.hotspot(td, pd, PRM, "center", 1, 6)
+    x = td
+    for _ in range(6):
+        x = P.hotspot(x, pd, PRM, "center", 1, 1)
+    assert torch.equal(fused, x)
