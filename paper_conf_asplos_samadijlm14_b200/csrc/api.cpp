@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -440,6 +441,15 @@ paraprox_status paraprox_tune_lattice(paraprox_filter f, const float* d_train, c
     return paraprox_tune_lattice_decide(parts, m, toq, out_scheme, out_reach, out_quality);
 }
 
+static bool hotspot_tb_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("PARAPROX_HOTSPOT_TB");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_scheme scheme, int reach,
                                  const float* d_temp, const float* d_power, float* d_out, const paraprox_image* img,
                                  int iterations, paraprox_stream s) {
@@ -492,6 +502,19 @@ paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_sc
         add.steps = iterations;
         cudaError_t e = launch_stencil(p, src, v0, d_out, img->pitch, ofs, cs, &add);
         if (e != cudaSuccess) return cuda_fail(e, "hotspot fused steps");
+        return PARAPROX_OK;
+    }
+    if (iterations > 1 && hotspot_tb_enabled()) {
+        // temporal blocking (k_hotspot.cu): up to 8 steps per HBM pass; the
+        // passes ping-pong so that the last lands in d_out
+        const int passes = (iterations + kHotspotMaxSteps - 1) / kHotspotMaxSteps;
+        for (int q = 0; q < passes; ++q) {
+            const int steps = std::min(kHotspotMaxSteps, iterations - q * kHotspotMaxSteps);
+            float* dst = ((passes - 1 - q) % 2 == 0) ? d_out : (float*)buf.p;
+            cudaError_t e = launch_hotspot_tb(p, src, d_power, dst, vn, ofs, add.alpha, add.beta, steps, cs);
+            if (e != cudaSuccess) return cuda_fail(e, "hotspot blocked steps");
+            src = dst;
+        }
         return PARAPROX_OK;
     }
     for (int it = 0; it < iterations; ++it) {

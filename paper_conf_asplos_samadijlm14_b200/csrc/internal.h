@@ -97,6 +97,12 @@ cudaError_t launch_stencil(const Plan& p, const float* in, const View& vin, floa
 // from the accessed rows/columns (reaches dy, dx); halos must be 0
 cudaError_t launch_lattice(const paraprox_filter_s& f, const float* in, const View& v, float* out,
                            long long out_pitch, long long out_fstride, int dy, int dx, cudaStream_t s);
+// temporally blocked HotSpot steps (k_hotspot.cu): `steps` <= kHotspotMaxSteps
+// steps of a 3x3 plan plus the power term in one pass; t, p, out share v's
+// layout (no halos)
+constexpr int kHotspotMaxSteps = 8;
+cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, float* out, const View& v,
+                              long long fs, float alpha, float beta, int steps, cudaStream_t s);
 cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
                            double* d_part3, double* d_scratch, cudaStream_t s);
 constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums
