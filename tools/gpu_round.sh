@@ -14,3 +14,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 600 --c
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_tiles|k_pointwise|k_lattice|k_quality_flat" -c 12 -o gpurun_out/prof_c2 -f python tools/prof_run.py --workload c2 --schemes exact:0,center:2,row:1 --lattice row:1,row:4 --quality --reps 2 > gpurun_out/ncu_c2.log 2>&1; echo ncu rc=$?
 fi
 cat gpurun_out/bench_c2.json
+timeout 900 python tools/toq_sweep.py > gpurun_out/toq_sweep.log 2>&1; echo sweep rc=$?
+timeout 400 python tools/kbench.py > gpurun_out/kbench.jsonl 2>&1; echo kbench rc=$?
+timeout 600 python tools/convsep.py > gpurun_out/convsep.log 2>&1; echo convsep rc=$?
+timeout 600 python tools/hotspot.py > gpurun_out/hotspot.log 2>&1; echo hotspot rc=$?
