@@ -675,34 +675,43 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     PPX_CUDA(scratch_alloc(&buf.p, sizeof(float) * 2 * plane * n, cs));
     float* din = (float*)buf.p;
     float* dout = din + plane * n;
-    // chunks: frames when batched, else row bands (halo rows come along)
-    // ~4 MiB per chunk (fill and drain of the copy pipeline are one chunk each), at most 32
+    // chunks: frames when batched, else row bands (halo rows come along);
+    // ~8 MiB per chunk (fill and drain of the copy pipeline are one chunk each), at most 16
     const long long total_bytes = (long long)sizeof(float) * plane * n;
-    const int want = (int)std::min<long long>(32, std::max<long long>(1, total_bytes >> 22));
+    const int want = (int)std::min<long long>(16, std::max<long long>(1, total_bytes >> 23));
     const int chunks = n > 1 ? std::min(n, want) : std::max(1, std::min(want, h / 64));
-    cudaStream_t up = nullptr, down = nullptr;
-    PPX_CUDA(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
-    cudaError_t err = cudaStreamCreateWithFlags(&down, cudaStreamNonBlocking);
-    if (err != cudaSuccess) {
-        cudaStreamDestroy(up);
-        return cuda_fail(err, "cudaStreamCreate");
+    // copy streams and events are created once per thread and device, reused
+    struct Pipe {
+        int dev = -1;
+        cudaStream_t up = nullptr, down = nullptr;
+        std::vector<cudaEvent_t> ev;
+    };
+    static thread_local Pipe pipe;
+    int dev = 0;
+    PPX_CUDA(cudaGetDevice(&dev));
+    if (pipe.dev != dev) {
+        if (pipe.up) cudaStreamDestroy(pipe.up);
+        if (pipe.down) cudaStreamDestroy(pipe.down);
+        for (auto& e : pipe.ev) cudaEventDestroy(e);
+        pipe = Pipe();
+        PPX_CUDA(cudaStreamCreateWithFlags(&pipe.up, cudaStreamNonBlocking));
+        PPX_CUDA(cudaStreamCreateWithFlags(&pipe.down, cudaStreamNonBlocking));
+        pipe.dev = dev;
     }
-    std::vector<cudaEvent_t> ev(3 * chunks + 1, nullptr);
-    for (auto& e : ev)
-        if (err == cudaSuccess) err = cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
-    auto cleanup = [&]() {
+    while ((int)pipe.ev.size() < 3 * chunks + 1) {
+        cudaEvent_t e;
+        PPX_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        pipe.ev.push_back(e);
+    }
+    cudaStream_t up = pipe.up, down = pipe.down;
+    std::vector<cudaEvent_t>& ev = pipe.ev;
+    cudaError_t err = cudaSuccess;
+    auto bail = [&](cudaError_t e2, const char* where) {
         cudaStreamSynchronize(down);
         cudaStreamSynchronize(up);
-        for (auto& e : ev)
-            if (e) cudaEventDestroy(e);
-        cudaStreamDestroy(up);
-        cudaStreamDestroy(down);
-    };
-    auto bail = [&](cudaError_t e2, const char* where) {
-        cleanup();
         return cuda_fail(e2, where);
     };
-    if (err != cudaSuccess) return bail(err, "cudaEventCreate");
+    const bool frames_contig = img->pitch == w && hfs == plane;
     // the device scratch is stream-ordered on cs: make the copy streams wait for it
     if ((err = cudaEventRecord(ev[3 * chunks], cs)) != cudaSuccess) return bail(err, "record");
     if ((err = cudaStreamWaitEvent(up, ev[3 * chunks], 0)) != cudaSuccess) return bail(err, "wait");
@@ -714,10 +723,16 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
         float* kout;
         if (n > 1) {
             const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
-            for (int fr = f0; fr < f1; ++fr)
-                if ((err = cudaMemcpy2DAsync(din + fr * plane, rowb, h_in + fr * hfs, sizeof(float) * img->pitch,
-                                             rowb, h, cudaMemcpyHostToDevice, up)) != cudaSuccess)
+            if (frames_contig) {
+                if ((err = cudaMemcpyAsync(din + f0 * plane, h_in + f0 * plane, sizeof(float) * plane * (f1 - f0),
+                                           cudaMemcpyHostToDevice, up)) != cudaSuccess)
                     return bail(err, "H2D");
+            } else {
+                for (int fr = f0; fr < f1; ++fr)
+                    if ((err = cudaMemcpy2DAsync(din + fr * plane, rowb, h_in + fr * hfs, sizeof(float) * img->pitch,
+                                                 rowb, h, cudaMemcpyHostToDevice, up)) != cudaSuccess)
+                        return bail(err, "H2D");
+            }
             v = {f1 - f0, h, w, (long long)w, plane, 0, h - 1};
             kin = din + f0 * plane;
             kout = dout + f0 * plane;
@@ -743,10 +758,16 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
         if ((err = cudaStreamWaitEvent(down, ev[3 * c + 1], 0)) != cudaSuccess) return bail(err, "wait");
         if (n > 1) {
             const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
-            for (int fr = f0; fr < f1; ++fr)
-                if ((err = cudaMemcpy2DAsync(h_out + fr * hfs, sizeof(float) * img->pitch, dout + fr * plane, rowb,
-                                             rowb, h, cudaMemcpyDeviceToHost, down)) != cudaSuccess)
+            if (frames_contig) {
+                if ((err = cudaMemcpyAsync(h_out + f0 * plane, dout + f0 * plane, sizeof(float) * plane * (f1 - f0),
+                                           cudaMemcpyDeviceToHost, down)) != cudaSuccess)
                     return bail(err, "D2H");
+            } else {
+                for (int fr = f0; fr < f1; ++fr)
+                    if ((err = cudaMemcpy2DAsync(h_out + fr * hfs, sizeof(float) * img->pitch, dout + fr * plane, rowb,
+                                                 rowb, h, cudaMemcpyDeviceToHost, down)) != cudaSuccess)
+                        return bail(err, "D2H");
+            }
         } else {
             const int r0 = (int)((long long)h * c / chunks), r1 = (int)((long long)h * (c + 1) / chunks);
             if ((err = cudaMemcpy2DAsync(h_out + (long long)r0 * img->pitch, sizeof(float) * img->pitch,
@@ -759,8 +780,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     if ((err = cudaEventRecord(ev[3 * chunks - 1], down)) != cudaSuccess) return bail(err, "record");
     if ((err = cudaStreamWaitEvent(cs, ev[3 * chunks - 1], 0)) != cudaSuccess) return bail(err, "wait");
     err = cudaStreamSynchronize(down);
-    cleanup();
-    if (err != cudaSuccess) return cuda_fail(err, "D2H sync");
+    if (err != cudaSuccess) return bail(err, "D2H sync");
     buf.p = nullptr;
     PPX_CUDA(cudaFreeAsync(din, cs));
     PPX_CUDA(cudaStreamSynchronize(cs));

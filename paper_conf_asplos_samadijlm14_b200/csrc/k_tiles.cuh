@@ -31,6 +31,13 @@
 #include "internal.h"
 #include "tma.cuh"
 
+#ifndef PPX_TILE_MAX_STAGES
+#define PPX_TILE_MAX_STAGES 3
+#endif
+#ifndef PPX_TILE_MIN_BLOCKS
+#define PPX_TILE_MIN_BLOCKS 2
+#endif
+
 namespace ppx {
 
 constexpr int kTW = 128;                 // tile width (outputs)
@@ -66,7 +73,7 @@ struct Geom {
     static constexpr int SH = kTH + 2 * HY;    // staged rows
     static constexpr int STAGE_BYTES = SW * SH * 4;
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
-    static constexpr int STAGES = (3 * STAGE_STRIDE <= 110 * 1024) ? 3 : 2;
+    static constexpr int STAGES = (3 * STAGE_STRIDE <= 110 * 1024 && PPX_TILE_MAX_STAGES >= 3) ? 3 : 2;
     static constexpr int SMEM = STAGES * STAGE_STRIDE;
 };
 
@@ -125,7 +132,7 @@ __device__ __forceinline__ void static_for(F&& f) {
 }
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
-__global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
                                                        const TileArgs A, const __grid_constant__ TapW W) {
     using G = Geom<HY, HX>;
     constexpr int HXP = G::HXP, SW = G::SW, SH = G::SH, NV = 4 + 2 * HXP;
@@ -198,28 +205,6 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
         }
 
         const int ty0 = wi * kRB;
-        // the additive input (HotSpot's power) is loaded before the compute so
-        // its latency hides behind the FMAs
-        const int xo = x0 + 4 * lane;
-        float4 pv[kRB];
-        if (A.addp) {
-            const float* abase = A.addp + (long long)f * A.afs + xo;
-#pragma unroll
-            for (int k = 0; k < kRB; ++k) {
-                const int y = y0 + ty0 + k;
-                pv[k] = make_float4(0.f, 0.f, 0.f, 0.f);
-                if (y < A.h && xo < A.w) {
-                    const float* ap = abase + (long long)y * A.apitch;
-                    if (xo + 3 < A.w) {
-                        pv[k] = __ldcs(reinterpret_cast<const float4*>(ap));
-                    } else {
-                        pv[k].x = ap[0];
-                        if (xo + 1 < A.w) pv[k].y = ap[1];
-                        if (xo + 2 < A.w) pv[k].z = ap[2];
-                    }
-                }
-            }
-        }
         // outputs as column pairs (c = 0,1 and 2,3): every FMA is a packed
         // FFMA2 (fma.rn.f32x2, sm_100) -- the same fp32 fma per lane, so the
         // per-pixel rounding and tap order are unchanged, at half the issue
@@ -303,8 +288,17 @@ __global__ void __launch_bounds__(kThreads, 2) k_tiles(const __grid_constant__ C
             if (y < A.h && x < A.w) {
                 float* o = obase + (long long)y * A.opitch;
                 float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
-                if (A.addp) {
-                    const float a4[4] = {pv[k].x, pv[k].y, pv[k].z, pv[k].w};
+                if (A.addp) {  // additive input (HotSpot's power, single steps and stripes)
+                    const float* ap = A.addp + (long long)f * A.afs + x + (long long)y * A.apitch;
+                    float a4[4] = {0.f, 0.f, 0.f, 0.f};
+                    if (x + 3 < A.w) {
+                        const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
+                        a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c)
+                            if (x + c < A.w) a4[c] = ap[c];
+                    }
 #pragma unroll
                     for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
                 }
