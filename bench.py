@@ -377,7 +377,16 @@ def main():
         scheme, reach, q_train = P.tune_decide(f, pt.cpu().numpy(), args.toq, wl["metric"])
     else:
         scheme, reach, q_train = P.tune(train, f, args.toq, wl["metric"])
-    tune_ms = 1e3 * (time.perf_counter() - t0)
+    tune_ms = 1e3 * (time.perf_counter() - t0)  # first call: includes one-time kernel setup
+    # warm: the tuner's throughput (exact once + every candidate scored by the
+    # fused stencil + quality kernels), device time on the stream
+    e_t0, e_t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e_t0.record(stream)
+    P.tune_partials(train, f, wl["metric"])
+    e_t1.record(stream)
+    torch.cuda.synchronize()
+    tune_warm_ms = e_t0.elapsed_time(e_t1)
+    n_cand = len(P.tune_candidates(f))
     train_keep = train
     plan = f.plan_info(*{"exact": (0, 0), "row": (reach, 0), "col": (0, reach),
                          "center": (reach, reach)}[scheme])
@@ -635,7 +644,9 @@ def main():
             "hbm_gbs": alg_bytes * ws / (ms_step * 1e-3) / 1e9,
             "tuned": {"scheme": scheme, "reach": reach, "quality_train": q_train, "quality_heldout": q_held,
                       "taps": plan["taps"], "halo_y": plan["halo_y"], "halo_x": plan["halo_x"],
-                      "tune_ms": tune_ms, "train_frames": tn},
+                      "tune_ms": tune_ms, "tune_warm_ms": tune_warm_ms, "candidates": n_cand,
+                      "tune_px_per_s": tn * th * tw * (1 + n_cand) / (tune_warm_ms * 1e-3),
+                      "train_frames": tn},
             "exact": {"value": exact_value, "unit": "Mpixel/s", "ms_per_step": exact_ms_step,
                       "hbm_gbs": alg_bytes * ws / (exact_ms_step * 1e-3) / 1e9,
                       "kernel_gbs": exact_achieved, "roofline_frac": exact_achieved / peak, "kernel": exact_kernel},

@@ -117,6 +117,15 @@ static const Plan& cand_plan(paraprox_filter f, const Candidate& c) {
     return is_skip_scheme(c.scheme) ? get_plan_skip(f, c.dy, c.dx) : get_plan(f, c.dy, c.dx);
 }
 
+bool fused_quality_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("PARAPROX_FUSED_QUALITY");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 constexpr int kMaxLatticeReach = 1 << 20;
 
 static paraprox_status run_lattice(paraprox_filter f, int dy, int dx, const float* in, float* out,
@@ -234,6 +243,15 @@ paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, cons
     cudaError_t e = launch_stencil(get_plan(f, 0, 0), d_train, vin, E, img->w, plane, cs);
     if (e != cudaSuccess) return cuda_fail(e, "exact launch");
     for (size_t k = 0; k < nc; ++k) {
+        // fused: the candidate's output is compared with E in the stencil's
+        // epilogue and never stored (8 B/px instead of 16)
+        bool fused = false;
+        if (fused_quality_enabled()) {
+            e = launch_stencil_quality(cand_plan(f, cands[k]), d_train, vin, E, img->w, plane, m, true,
+                                       parts + 3 * k, scratch, cs, &fused);
+            if (e != cudaSuccess) return cuda_fail(e, "fused candidate launch");
+        }
+        if (fused) continue;
         e = launch_stencil(cand_plan(f, cands[k]), d_train, vin, A, img->w, plane, cs);
         if (e != cudaSuccess) return cuda_fail(e, "candidate launch");
         e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);

@@ -19,6 +19,17 @@ cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float*
                            long long ofs, cudaStream_t s, const Addend* add);
 cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, float* out, long long opitch,
                              long long ofs, cudaStream_t s, const Addend* add);
+bool launch_pointwise_quality(const Plan& p, const float* in, const View& v, const float* ref, long long rpitch,
+                              long long rfs, int metric, int ref_exact, double* part, int* grid_out, cudaStream_t s,
+                              cudaError_t* err);
+
+struct QualityOut {
+    const float* ref;
+    long long rpitch, rfs;
+    int metric, ref_exact;
+    double* part;
+    int grid;  // written: CTAs that wrote partials
+};
 
 void register_r1_dense();
 void register_r2_dense();
@@ -83,7 +94,8 @@ void register_tile_instance(const TileInstance& ti) {
 }
 
 static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const View& v, float* out,
-                                long long opitch, long long ofs, cudaStream_t s, const Addend* add, bool* taken) {
+                                long long opitch, long long ofs, cudaStream_t s, const Addend* add, bool* taken,
+                                QualityOut* qo = nullptr) {
     *taken = false;
     int dev = 0;
     cudaError_t err = cudaGetDevice(&dev);
@@ -134,6 +146,14 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.afs = add ? add->fstride : 0;
     A.alpha = add ? add->alpha : 0.f;
     A.beta = add ? add->beta : 0.f;
+    A.refp = qo ? qo->ref : nullptr;
+    A.rpitch = qo ? qo->rpitch : 0;
+    A.rfs = qo ? qo->rfs : 0;
+    A.metric = qo ? qo->metric : 0;
+    A.ref_exact = qo ? qo->ref_exact : 0;
+    A.part = qo ? qo->part : nullptr;
+    if (qo && ((reinterpret_cast<uintptr_t>(qo->ref) & 15) || (qo->rpitch & 3) || (v.n > 1 && (qo->rfs & 3))))
+        return cudaSuccess;
     TapW W = {};
     if (p.separable) {
         for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 8] = p.wyf[i];
@@ -142,8 +162,10 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
         for (int i = 0; i < p.ny; ++i)
             for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];
     }
-    const long long cap = (long long)g_sms[dev] * e.occ[dev];
+    long long cap = (long long)g_sms[dev] * e.occ[dev];
+    if (qo && cap > kQualityBlocks) cap = kQualityBlocks;  // one partial pair per CTA
     const int grid = (int)(nt < cap ? nt : cap);
+    if (qo) qo->grid = grid;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(kThreads);
@@ -156,7 +178,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     cfg.numAttrs = 1;
     err = cudaLaunchKernelEx(&cfg, e.ti.fn, tmap, A, W);
     if (err != cudaSuccess) return err;
-    count_launch(e.ti.name);
+    count_launch(qo ? "tile_quality" : e.ti.name);
     *taken = true;
     return cudaGetLastError();
 }
@@ -177,6 +199,40 @@ cudaError_t launch_stencil(const Plan& p, const float* in, const View& v, float*
         }
     }
     return launch_generic(p, in, v, out, opitch, ofs, s, add);
+}
+
+cudaError_t launch_stencil_quality(const Plan& p, const float* in, const View& v, const float* ref,
+                                   long long ref_pitch, long long ref_fstride, paraprox_metric m, bool ref_exact,
+                                   double* d_part3, double* d_scratch, cudaStream_t s, bool* fused) {
+    *fused = false;
+    if (force_generic()) return cudaSuccess;
+    const double count = (double)v.n * (double)v.h * (double)v.w;
+    if (p.hy == 0 && p.hx == 0) {
+        int grid = 0;
+        cudaError_t err = cudaSuccess;
+        if (!launch_pointwise_quality(p, in, v, ref, ref_pitch, ref_fstride, (int)m, ref_exact ? 1 : 0, d_scratch,
+                                      &grid, s, &err))
+            return cudaSuccess;
+        if (err != cudaSuccess) return err;
+        *fused = true;
+        return launch_quality_final(d_scratch, grid, count, m, d_part3, s);
+    }
+    const int rmax = p.separable ? 8 : 4;
+    if (p.ry > rmax || p.rx > rmax) return cudaSuccess;
+    init_registry();
+    for (Entry& e : reg()) {
+        if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;
+        QualityOut qo{ref, ref_pitch, ref_fstride, (int)m, ref_exact ? 1 : 0, d_scratch, 0};
+        bool taken = false;
+        // the output pointer only fixes the layout checks: nothing is stored
+        cudaError_t err = launch_tiles(e, p, in, v, const_cast<float*>(ref), ref_pitch, ref_fstride, s, nullptr,
+                                       &taken, &qo);
+        if (err != cudaSuccess) return err;
+        if (!taken) return cudaSuccess;
+        *fused = true;
+        return launch_quality_final(d_scratch, qo.grid, count, m, d_part3, s);
+    }
+    return cudaSuccess;
 }
 
 }  // namespace ppx

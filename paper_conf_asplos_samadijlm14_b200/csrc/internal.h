@@ -103,6 +103,17 @@ cudaError_t launch_lattice(const paraprox_filter_s& f, const float* in, const Vi
 constexpr int kHotspotMaxSteps = 8;
 cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, float* out, const View& v,
                               long long fs, float alpha, float beta, int steps, cudaStream_t s);
+// Fused stencil + quality (the tuner's candidates, the runtime's checks): the
+// plan's output is compared with `ref` (laid out like the output; ref_exact:
+// ref holds the exact output, else the approximation) instead of being
+// stored; 3 partials at d_part3 as launch_quality writes them.  *fused =
+// false (nothing launched) when no fused kernel takes the plan and layout.
+cudaError_t launch_stencil_quality(const Plan& p, const float* in, const View& vin, const float* ref,
+                                   long long ref_pitch, long long ref_fstride, paraprox_metric m, bool ref_exact,
+                                   double* d_part3, double* d_scratch, cudaStream_t s, bool* fused);
+bool fused_quality_enabled();  // PARAPROX_FUSED_QUALITY=0 turns the fused paths off
+cudaError_t launch_quality_final(const double* d_scratch, int g, double count, paraprox_metric m, double* d_part3,
+                                 cudaStream_t s);
 cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
                            double* d_part3, double* d_scratch, cudaStream_t s);
 constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums

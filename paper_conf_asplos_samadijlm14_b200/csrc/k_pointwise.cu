@@ -10,7 +10,9 @@
 //
 // Rounding matches the tile kernels bit for bit: dense fmaf(w, x, 0);
 // separable fmaf(wy, fmaf(wx, x, 0), 0) (horizontal, then vertical pass).
-#include "internal.h"
+#include <algorithm>
+
+#include "quality.cuh"
 
 namespace ppx {
 
@@ -74,6 +76,49 @@ __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict_
     if (blockIdx.x == 0)
         for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x)
             out[x] = add.p ? steps1<SEP>(in[x], add.p[x], w0, w1, add) : pw<SEP>(in[x], w0, w1);
+}
+
+// fused quality (the tuner's centre candidates): compare w' x with the
+// reference instead of storing; 2 fp64 partials per CTA, deterministic order
+template <bool SEP>
+__global__ void __launch_bounds__(256) k_pointwise_flat_q(const float* __restrict__ in, const float* __restrict__ ref,
+                                                          long long count, float w0, float w1, int metric,
+                                                          int ref_exact, double* __restrict__ part) {
+    const long long n4 = count >> 2;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const float4* i4 = reinterpret_cast<const float4*>(in);
+    const float4* r4 = reinterpret_cast<const float4*>(ref);
+    RAcc q;
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    auto term = [&](float v, float r) { q.add(metric, ref_exact ? r : v, ref_exact ? v : r); };
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kPU * stride) {
+        float4 v[kPU], r[kPU];
+#pragma unroll
+        for (int u = 0; u < kPU; ++u)
+            if (i + u * stride < n4) {
+                v[u] = __ldcs(i4 + i + u * stride);
+                r[u] = __ldcs(r4 + i + u * stride);
+            }
+#pragma unroll
+        for (int u = 0; u < kPU; ++u)
+            if (i + u * stride < n4) {
+                const float4 a = pw4<SEP>(v[u], w0, w1);
+                term(a.x, r[u].x);
+                term(a.y, r[u].y);
+                term(a.z, r[u].z);
+                term(a.w, r[u].w);
+            }
+    }
+    if (blockIdx.x == 0)
+        for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) term(pw<SEP>(in[x], w0, w1), ref[x]);
+    double s0, s1;
+    q.get(metric, s0, s1);
+    block_sum2(s0, s1);
+    if (threadIdx.x == 0) {
+        part[2 * blockIdx.x] = s0;
+        part[2 * blockIdx.x + 1] = s1;
+    }
 }
 
 // any layout: rows of the output image, 128-bit where both rows allow it
@@ -150,6 +195,39 @@ cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, floa
     }
     if (err != cudaSuccess) return err;
     return cudaGetLastError();
+}
+
+}  // namespace ppx
+
+namespace ppx {
+
+// the map kernel in fused-quality mode; false when the layout is not flat
+bool launch_pointwise_quality(const Plan& p, const float* in, const View& v, const float* ref, long long rpitch,
+                              long long rfs, int metric, int ref_exact, double* part, int* grid_out, cudaStream_t s,
+                              cudaError_t* err) {
+    const long long count = (long long)v.n * v.h * v.w;
+    const bool flat = v.pitch == v.w && rpitch == v.w && (v.n == 1 || (v.fstride == (long long)v.h * v.w &&
+                      rfs == (long long)v.h * v.w)) && v.lo == 0 &&
+                      (((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(ref)) & 15) == 0);
+    if (!flat) return false;
+    int dev = 0, nsm = 148;
+    *err = cudaGetDevice(&dev);
+    if (*err != cudaSuccess) return true;
+    *err = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (*err != cudaSuccess) return true;
+    const float w0 = p.separable ? p.wyf[0] : p.wf[0];
+    const float w1 = p.separable ? p.wxf[0] : 1.f;
+    const long long want = (count / 4 + 255) / 256;
+    long long grid = std::min<long long>((long long)nsm * 8, kQualityBlocks);
+    grid = std::max<long long>(1, std::min(grid, want));
+    if (p.separable)
+        k_pointwise_flat_q<true><<<(unsigned)grid, 256, 0, s>>>(in, ref, count, w0, w1, metric, ref_exact, part);
+    else
+        k_pointwise_flat_q<false><<<(unsigned)grid, 256, 0, s>>>(in, ref, count, w0, w1, metric, ref_exact, part);
+    count_launch(p.separable ? "sep_map_quality" : "dense_map_quality");
+    *grid_out = (int)grid;
+    *err = cudaGetLastError();
+    return true;
 }
 
 }  // namespace ppx

@@ -6,115 +6,9 @@
 // (kQualityBlocks, or fewer rows), each walking its rows in a fixed order,
 // fixed warp-shuffle trees, then one CTA summing the per-CTA partials in a
 // fixed order.  No atomics.  8 bytes of HBM read per pixel, nothing written.
-#include "internal.h"
+#include "quality.cuh"
 
 namespace ppx {
-
-// Per-thread accumulators.  L2 / PSNR: fp64 (the difference of two fp32
-// values is exact in fp64; 2 DFMA per pixel).  MRE needs a quotient per
-// pixel, and fp64 division is far below the HBM rate on this part (the first
-// version ran at ~1.5 TB/s), so each term |A-E|/|E| is formed as an unevaluated
-// fp32 pair q0 + q1 (exact difference by TwoSum, quotient by the approximate
-// fp32 reciprocal plus one FMA remainder correction, relative error ~2^-46)
-// whose two parts are summed in two fp64 accumulators.  Terms the pair arithmetic cannot carry (|E| tiny, |A-E| huge) take
-// the fp64 path.  Tests bound the result against the fp64 oracle at 1e-12.
-template <int M>
-struct QAcc {
-    double s0 = 0.0, s1 = 0.0;
-    bool bad = false;                                       // never set: no fix-up pass
-    __device__ __forceinline__ void fix(float, float) {}
-    __device__ __forceinline__ void add(float e, float a) {
-        const double de = (double)e, da = (double)a;
-        const double d = da - de;
-        if (M == PARAPROX_L2) {
-            s0 = fma(d, d, s0);
-            s1 = fma(de, de, s1);
-        } else {
-            s0 = fma(d, d, s0);
-        }
-    }
-    __device__ __forceinline__ void get(double& a, double& b) const {
-        a = s0;
-        b = s1;
-    }
-};
-
-__device__ __forceinline__ void two_sum(float a, float b, float& s, float& err) {
-    s = __fadd_rn(a, b);
-    const float bb = __fsub_rn(s, a);
-    err = __fadd_rn(__fsub_rn(a, __fsub_rn(s, bb)), __fsub_rn(b, bb));
-}
-
-__device__ __forceinline__ float rcp_approx(float x) {
-    float r;
-    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
-    return r;
-}
-
-template <>
-struct QAcc<PARAPROX_MRE> {
-    double hi = 0.0, lo = 0.0;  // sums of the leading and trailing parts of the terms
-    bool bad = false;  // a term the pair arithmetic cannot carry was skipped
-    // the fast path skips terms with |E| tiny or huge or |A-E| huge (and the
-    // E == 0 convention, S12); a second pass adds exactly those in fp64
-    __device__ __forceinline__ static bool fast_ok(float ae, float dh) {
-        return ae >= 1e-30f && ae <= 1e30f && fabsf(dh) <= 1e30f;
-    }
-    __device__ __forceinline__ void add(float e, float a) {
-        float dh, dl;
-        two_sum(a, -e, dh, dl);  // A - E exactly, as dh + dl
-        const float ae = fabsf(e);
-        const bool ok = fast_ok(ae, dh);
-        bad |= !ok;
-        if (dh < 0.f) {
-            dh = -dh;
-            dl = -dl;
-        }
-        // q0 + q1 = |A-E| / |E| to ~2^-46: the remainder of the first quotient
-        // is exact under the FMA, so the approximate reciprocal's own error is
-        // corrected by the second term
-        const float rc = rcp_approx(ae);
-        const float q0 = __fmul_rn(dh, rc);
-        const float rem = __fadd_rn(__fmaf_rn(-q0, ae, dh), dl);
-        hi += ok ? (double)q0 : 0.0;
-        lo += ok ? (double)__fmul_rn(rem, rc) : 0.0;
-    }
-    __device__ __forceinline__ void fix(float e, float a) {
-        float dh, dl;
-        two_sum(a, -e, dh, dl);
-        if (!fast_ok(fabsf(e), dh)) {
-            const double de = (double)e, da = (double)a;
-            hi += de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
-        }
-    }
-    __device__ __forceinline__ void get(double& a, double& b) const {
-        a = hi + lo;
-        b = 0.0;
-    }
-};
-
-__device__ __forceinline__ void block_sum2(double& s0, double& s1) {
-    __shared__ double red[2][32];
-    for (int o = 16; o > 0; o >>= 1) {
-        s0 += __shfl_down_sync(0xffffffffu, s0, o);
-        s1 += __shfl_down_sync(0xffffffffu, s1, o);
-    }
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (lane == 0) {
-        red[0][warp] = s0;
-        red[1][warp] = s1;
-    }
-    __syncthreads();
-    if (warp == 0) {
-        const int nw = blockDim.x >> 5;
-        s0 = lane < nw ? red[0][lane] : 0.0;
-        s1 = lane < nw ? red[1][lane] : 0.0;
-        for (int o = 16; o > 0; o >>= 1) {
-            s0 += __shfl_down_sync(0xffffffffu, s0, o);
-            s1 += __shfl_down_sync(0xffffffffu, s1, o);
-        }
-    }
-}
 
 // Contiguous images (pitch == w, frames back to back) are one flat array:
 // each thread keeps kQU independent 128-bit loads of E and of A in flight per
@@ -266,6 +160,17 @@ cudaError_t launch_quality(const float* e, const float* a, const View& v, parapr
     }
 #undef PPX_QUALITY_CASE
     count_launch(flat ? "quality_flat" : "quality_partials");
+    count_launch("quality_final");
+    return cudaGetLastError();
+}
+
+cudaError_t launch_quality_final(const double* d_scratch, int g, double count, paraprox_metric m, double* d_part3,
+                                 cudaStream_t s) {
+    switch (m) {
+    case PARAPROX_MRE: k_quality_final<PARAPROX_MRE><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
+    case PARAPROX_L2: k_quality_final<PARAPROX_L2><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
+    default: k_quality_final<PARAPROX_PSNR><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
+    }
     count_launch("quality_final");
     return cudaGetLastError();
 }

@@ -29,6 +29,7 @@
 #include <utility>
 
 #include "internal.h"
+#include "quality.cuh"
 #include "tma.cuh"
 
 #ifndef PPX_TILE_MAX_STAGES
@@ -62,6 +63,12 @@ struct TileArgs {
     const float* addp;  // optional additive input (NEXT-4): out += alpha * addp + beta
     long long apitch, afs;
     float alpha, beta;
+    // optional fused quality (the tuner's candidates, the runtime's checks):
+    // instead of storing, compare with refp and write 2 fp64 partials per CTA
+    const float* refp;
+    long long rpitch, rfs;
+    int metric, ref_exact;  // ref_exact: refp holds the exact output (else the approximation)
+    double* part;
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -175,6 +182,7 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             if (t < A.ntiles) issue(t, s);
         }
 
+    RAcc racc;  // fused-quality partials (A.refp)
     int it = 0;
     for (int tile = blockIdx.x; tile < A.ntiles; tile += gridDim.x, ++it) {
         const int s = it % G::STAGES;
@@ -302,7 +310,22 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
 #pragma unroll
                     for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
                 }
-                if (x + 3 < A.w) {
+                if (A.refp) {  // fused quality: no store
+                    const float* rp = A.refp + (long long)f * A.rfs + x + (long long)y * A.rpitch;
+                    float q4[4] = {0.f, 0.f, 0.f, 0.f};
+                    if (x + 3 < A.w) {
+                        const float4 t = __ldcs(reinterpret_cast<const float4*>(rp));
+                        q4[0] = t.x, q4[1] = t.y, q4[2] = t.z, q4[3] = t.w;
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c)
+                            if (x + c < A.w) q4[c] = rp[c];
+                    }
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (x + c < A.w)
+                            racc.add(A.metric, A.ref_exact ? q4[c] : r4[c], A.ref_exact ? r4[c] : q4[c]);
+                } else if (x + 3 < A.w) {
                     __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
                 } else {
 #pragma unroll
@@ -312,6 +335,15 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             }
         }
         __syncthreads();  // stage s fully consumed before it is refilled
+    }
+    if (A.refp) {  // deterministic: fixed tile order per CTA, fixed reduction tree
+        double s0, s1;
+        racc.get(A.metric, s0, s1);
+        block_sum2(s0, s1);
+        if (tid == 0) {
+            A.part[2 * blockIdx.x] = s0;
+            A.part[2 * blockIdx.x + 1] = s1;
+        }
     }
 }
 

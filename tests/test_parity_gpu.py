@@ -284,3 +284,40 @@ def test_generic_and_tile_kernels_bitwise(P, w):
         # centre-only plans are maps: the misaligned copy takes the row-wise map
         assert ka != "generic" and kb in ("generic", "dense_map_rows"), (ka, kb)
         assert torch.equal(a, b), (dy, dx)
+
+
+def test_fused_tuner_partials_match_unfused(P):
+    """The tuner scores candidates with the fused stencil + quality epilogue;
+    the unfused path (PARAPROX_FUSED_QUALITY=0: stencil stored, then the
+    quality kernel) gives the same qualities to rounding and the same
+    decisions."""
+    import json
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import json, sys, torch
+sys.path.insert(0, %r)
+import paper_conf_asplos_samadijlm14_b200 as pkg
+import workloads as W
+from workloads import filters as F
+P = pkg.paraprox
+out = {}
+for name, w, m in [("mean5", F.mean(5), "mre"), ("conv9", F.conv(9), "l2"), ("sep7", F.separable(7), "l2")]:
+    f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+    x = torch.from_numpy(W.frames(4, 160, 200, 3)).cuda()
+    out[name] = P.tune_partials(x, f, m).tolist()
+print(json.dumps(out))
+''' % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))),)
+    res = {}
+    for flag in ("1", "0"):
+        env = dict(os.environ, PARAPROX_FUSED_QUALITY=flag)
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr
+        res[flag] = json.loads(r.stdout.strip().splitlines()[-1])
+    metric = {"mean5": "mre", "conv9": "l2", "sep7": "l2"}
+    for name in res["1"]:
+        a, b = np.array(res["1"][name]), np.array(res["0"][name])
+        qa = [P.quality_from_partials(a[3 * k:3 * k + 3], metric[name]) for k in range(len(a) // 3)]
+        qb = [P.quality_from_partials(b[3 * k:3 * k + 3], metric[name]) for k in range(len(b) // 3)]
+        np.testing.assert_allclose(qa, qb, rtol=0, atol=1e-12)
