@@ -279,10 +279,22 @@ def run_stripes(args, dist, rank, ws, local):
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
         return float(tot[0]) / args.steps, launches
 
+    if args.halo == "peer":
+        # the neighbours' boundary rows are read inside the stencil kernel
+        # through CUDA IPC mappings (NVLink P2P): no collective per step
+        ps = D.PeerStripe(s, wd, dev)
+        ps.buf.copy_(buf[s.cap:s.cap + s.rows])
+        del buf
+        ps.ready()
+        step_approx = lambda: ps.stencil(f, scheme, reach, out)  # noqa: E731
+        step_exact = lambda: ps.stencil(f, "exact", 0, out)  # noqa: E731
+    else:
+        step_approx = lambda: D.stencil_stripe(buf, s, f, scheme, reach, out)  # noqa: E731
+        step_exact = lambda: D.stencil_stripe(buf, s, f, "exact", 0, out)  # noqa: E731
     with ClockSampler(local) as clk:
-        ms, launches = timed(lambda: D.stencil_stripe(buf, s, f, scheme, reach, out))
+        ms, launches = timed(step_approx)
         approx_kernel = P.last_kernel()
-        ex_ms, _ = timed(lambda: D.stencil_stripe(buf, s, f, "exact", 0, out))
+        ex_ms, _ = timed(step_exact)
     peak, peak_kind = load_peaks()
     local_bytes = 8.0 * s.rows * wd
     if rank == 0:
@@ -292,7 +304,9 @@ def run_stripes(args, dist, rank, ws, local):
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "c4", "desc": wl["desc"] + ", row stripes", "h": h, "w": wd, "filter": "conv9",
                        "toq": args.toq, "metric_quality": wl["metric"],
-                       "parallelism": f"row stripes x{ws}: {s.rows} rows per rank, NCCL halo send/recv of h_y rows",
+                       "parallelism": (f"row stripes x{ws}: {s.rows} rows per rank, h_y halo rows read in-kernel "
+                                       f"from the neighbours over CUDA IPC / NVLink" if args.halo == "peer" else
+                                       f"row stripes x{ws}: {s.rows} rows per rank, NCCL halo send/recv of h_y rows"),
                        "l2_defeat": "inputs larger than L2 (a stripe is >= 512 MiB)"},
             "tuned": {"scheme": scheme, "reach": reach, "quality_train": q_train, "tune_ms": tune_ms,
                       "halo_y": hy, "halo_bytes_per_step_per_neighbour": hy * wd * 4},
@@ -308,6 +322,8 @@ def run_stripes(args, dist, rank, ws, local):
         }
         print(json.dumps(line), flush=True)
     dist.barrier()
+    if args.halo == "peer":
+        ps.close()
     dist.destroy_process_group()
 
 
@@ -323,6 +339,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-lattice", action="store_true")
     ap.add_argument("--no-graph", action="store_true", help="time the eager ctypes loop instead of CUDA graphs")
+    ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
+                    help="c4 row stripes at N>1: halo rows read in-kernel over IPC/NVLink, or NCCL send/recv")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":

@@ -164,6 +164,27 @@ PARAPROX_API paraprox_status paraprox_stencil_skip_xy(paraprox_filter f, int ski
                                          const float* d_in, float* d_out,
                                          const paraprox_image* img, paraprox_stream s);
 
+/* Row stripe with peer halos (§8(e) P2; the B200-native form of the halo
+ * exchange): the stencil of one stripe (img: n == 1, no halos) whose top_rows
+ * rows directly above row 0 are read from d_top and bot_rows rows below row
+ * h-1 from d_bot (pitch src_pitch elements) -- device pointers that may map a
+ * neighbouring GPU's stripe over NVLink (paraprox_ipc_open), read inside the
+ * stencil kernel with no separate collective.  0 rows = the image edge
+ * (clamp).  Only the plan's halo h_y rows are read.  The caller orders the
+ * neighbours' writes before this call (e.g. a barrier).  Asynchronous on s. */
+PARAPROX_API paraprox_status paraprox_stencil_peer(paraprox_filter f, paraprox_scheme scheme, int reach,
+                                      const float* d_in, float* d_out, const paraprox_image* img,
+                                      const float* d_top, int top_rows, const float* d_bot, int bot_rows,
+                                      long long src_pitch, paraprox_stream s);
+
+/* CUDA IPC of device buffers between the processes of one node (one per GPU):
+ * export writes a 64-byte handle of the allocation containing d_ptr and
+ * d_ptr's byte offset in it; open maps a peer's handle (peer access enabled
+ * lazily) and returns the allocation's base; close unmaps it. */
+PARAPROX_API paraprox_status paraprox_ipc_export(const void* d_ptr, void* h_handle64, long long* offset);
+PARAPROX_API paraprox_status paraprox_ipc_open(const void* h_handle64, void** d_base);
+PARAPROX_API paraprox_status paraprox_ipc_close(void* d_base);
+
 /* End-to-end convenience over HOST buffers: copies h_in to the device,
  * runs the stencil (scheme, reach), copies the result to h_out, overlapping
  * the transfers with the kernels chunk by chunk.  Pinned host memory gives

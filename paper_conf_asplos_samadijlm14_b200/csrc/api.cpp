@@ -1,6 +1,8 @@
 // api.cpp -- the extern "C" entry points of libparaprox (include/paraprox.h):
 // argument validation, plan lookup, stream-ordered scratch, the TOQ tuner and
 // the host-buffer end-to-end path.  All arithmetic runs in the kernels.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -541,6 +543,99 @@ paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_sc
         if (e != cudaSuccess) return cuda_fail(e, "hotspot step");
         src = dst;
     }
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_stencil_peer(paraprox_filter f, paraprox_scheme scheme, int reach, const float* d_in,
+                                      float* d_out, const paraprox_image* img, const float* d_top, int top_rows,
+                                      const float* d_bot, int bot_rows, long long src_pitch, paraprox_stream s) {
+    if (!f || !d_in || !d_out || !img) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0 || top_rows < 0 || bot_rows < 0) return fail(PARAPROX_ERR_INVALID_ARG, "negative reach or rows");
+    if ((top_rows && !d_top) || (bot_rows && !d_bot)) return fail(PARAPROX_ERR_INVALID_ARG, "NULL halo source");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    if (img->n != 1) return fail(PARAPROX_ERR_INVALID_ARG, "peer halos need n == 1");
+    if ((top_rows || bot_rows) && src_pitch < img->w) return fail(PARAPROX_ERR_INVALID_ARG, "src_pitch < w");
+    if (overlaps(d_in, d_out, img)) return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps d_in");
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    const Plan& p = get_plan(f, dy, dx);
+    const int ntop = std::min(top_rows, p.hy), nbot = std::min(bot_rows, p.hy);
+    cudaStream_t cs = (cudaStream_t)s;
+    const View v = view_of(img);
+    if (ntop == 0 && nbot == 0) {  // nothing to read from the neighbours
+        cudaError_t e = launch_stencil(p, d_in, v, d_out, img->pitch, (long long)img->h * img->pitch, cs);
+        if (e != cudaSuccess) return cuda_fail(e, "stencil launch");
+        return PARAPROX_OK;
+    }
+    bool taken = false;
+    cudaError_t e = launch_stencil_peer(p, d_in, v, d_out, img->pitch, d_top + (long long)(top_rows - ntop) * src_pitch,
+                                        ntop, d_bot, nbot, src_pitch, cs, &taken);
+    if (e != cudaSuccess) return cuda_fail(e, "peer stencil launch");
+    if (taken) return PARAPROX_OK;
+    // fallback: gather the halo rows next to a copy of the stripe, then the
+    // regular halo path (peer rows are read by the copy engine)
+    const long long rows = (long long)ntop + img->h + nbot;
+    DevBuf buf;
+    buf.s = cs;
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(float) * rows * img->w, cs));
+    float* g = (float*)buf.p;
+    const size_t rowb = sizeof(float) * img->w;
+    if (ntop)
+        PPX_CUDA(cudaMemcpy2DAsync(g, rowb, d_top + (long long)(top_rows - ntop) * src_pitch, sizeof(float) * src_pitch,
+                                   rowb, ntop, cudaMemcpyDefault, cs));
+    PPX_CUDA(cudaMemcpy2DAsync(g + (long long)ntop * img->w, rowb, d_in, sizeof(float) * img->pitch, rowb, img->h,
+                               cudaMemcpyDefault, cs));
+    if (nbot)
+        PPX_CUDA(cudaMemcpy2DAsync(g + (long long)(ntop + img->h) * img->w, rowb, d_bot, sizeof(float) * src_pitch, rowb,
+                                   nbot, cudaMemcpyDefault, cs));
+    View vg;
+    vg.n = 1;
+    vg.h = img->h;
+    vg.w = img->w;
+    vg.pitch = img->w;
+    vg.fstride = rows * img->w;
+    vg.lo = -ntop;
+    vg.hi = img->h - 1 + nbot;
+    e = launch_stencil(p, g + (long long)ntop * img->w, vg, d_out, img->pitch, (long long)img->h * img->pitch, cs);
+    if (e != cudaSuccess) return cuda_fail(e, "stencil launch");
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_ipc_export(const void* d_ptr, void* h_handle, long long* offset) {
+    if (!d_ptr || !h_handle || !offset) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    static PFN_cuMemGetAddressRange_v3020 range = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            range = reinterpret_cast<PFN_cuMemGetAddressRange_v3020>(fn);
+    });
+    if (!range) return fail(PARAPROX_ERR_CUDA, "cuMemGetAddressRange unavailable");
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (CUdeviceptr)d_ptr) != CUDA_SUCCESS) return fail(PARAPROX_ERR_CUDA, "cuMemGetAddressRange");
+    cudaIpcMemHandle_t h;
+    PPX_CUDA(cudaIpcGetMemHandle(&h, (void*)base));
+    std::memcpy(h_handle, &h, sizeof(h));
+    *offset = (long long)((CUdeviceptr)d_ptr - base);
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_ipc_open(const void* h_handle, void** d_base) {
+    if (!h_handle || !d_base) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, h_handle, sizeof(h));
+    PPX_CUDA(cudaIpcOpenMemHandle(d_base, h, cudaIpcMemLazyEnablePeerAccess));
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_ipc_close(void* d_base) {
+    if (!d_base) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    PPX_CUDA(cudaIpcCloseMemHandle(d_base));
     return PARAPROX_OK;
 }
 

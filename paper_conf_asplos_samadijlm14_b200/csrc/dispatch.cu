@@ -23,6 +23,13 @@ bool launch_pointwise_quality(const Plan& p, const float* in, const View& v, con
                               long long rfs, int metric, int ref_exact, double* part, int* grid_out, cudaStream_t s,
                               cudaError_t* err);
 
+struct PeerHalo {
+    const float* top;
+    const float* bot;
+    int ntop, nbot;
+    long long pitch;
+};
+
 struct QualityOut {
     const float* ref;
     long long rpitch, rfs;
@@ -95,7 +102,7 @@ void register_tile_instance(const TileInstance& ti) {
 
 static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const View& v, float* out,
                                 long long opitch, long long ofs, cudaStream_t s, const Addend* add, bool* taken,
-                                QualityOut* qo = nullptr) {
+                                QualityOut* qo = nullptr, const PeerHalo* ph = nullptr) {
     *taken = false;
     int dev = 0;
     cudaError_t err = cudaGetDevice(&dev);
@@ -152,6 +159,11 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.metric = qo ? qo->metric : 0;
     A.ref_exact = qo ? qo->ref_exact : 0;
     A.part = qo ? qo->part : nullptr;
+    A.htop = ph ? ph->top : nullptr;
+    A.hbot = ph ? ph->bot : nullptr;
+    A.ntop = ph ? ph->ntop : 0;
+    A.nbot = ph ? ph->nbot : 0;
+    A.hpitch = ph ? ph->pitch : 0;
     if (qo && ((reinterpret_cast<uintptr_t>(qo->ref) & 15) || (qo->rpitch & 3) || (v.n > 1 && (qo->rfs & 3))))
         return cudaSuccess;
     TapW W = {};
@@ -231,6 +243,22 @@ cudaError_t launch_stencil_quality(const Plan& p, const float* in, const View& v
         if (!taken) return cudaSuccess;
         *fused = true;
         return launch_quality_final(d_scratch, qo.grid, count, m, d_part3, s);
+    }
+    return cudaSuccess;
+}
+
+cudaError_t launch_stencil_peer(const Plan& p, const float* in, const View& v, float* out, long long opitch,
+                                const float* htop, int ntop, const float* hbot, int nbot, long long hpitch,
+                                cudaStream_t s, bool* taken) {
+    *taken = false;
+    if (force_generic() || v.n != 1 || v.lo != 0 || v.hi != v.h - 1) return cudaSuccess;
+    const int rmax = p.separable ? 8 : 4;
+    if (p.ry > rmax || p.rx > rmax) return cudaSuccess;
+    init_registry();
+    const PeerHalo ph{htop, hbot, ntop, nbot, hpitch};
+    for (Entry& e : reg()) {
+        if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;
+        return launch_tiles(e, p, in, v, out, opitch, (long long)v.h * opitch, s, nullptr, taken, nullptr, &ph);
     }
     return cudaSuccess;
 }

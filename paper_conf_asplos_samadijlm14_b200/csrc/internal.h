@@ -111,6 +111,12 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
 cudaError_t launch_stencil_quality(const Plan& p, const float* in, const View& vin, const float* ref,
                                    long long ref_pitch, long long ref_fstride, paraprox_metric m, bool ref_exact,
                                    double* d_part3, double* d_scratch, cudaStream_t s, bool* fused);
+// Row-stripe stencil whose halo rows are read inside the kernel from peer
+// pointers (CUDA IPC mappings of the neighbours' stripes): *taken = false
+// when no tile instance takes the plan (the caller falls back to staging).
+cudaError_t launch_stencil_peer(const Plan& p, const float* in, const View& v, float* out, long long opitch,
+                                const float* htop, int ntop, const float* hbot, int nbot, long long hpitch,
+                                cudaStream_t s, bool* taken);
 bool fused_quality_enabled();  // PARAPROX_FUSED_QUALITY=0 turns the fused paths off
 cudaError_t launch_quality_final(const double* d_scratch, int g, double count, paraprox_metric m, double* d_part3,
                                  cudaStream_t s);

@@ -69,6 +69,14 @@ struct TileArgs {
     long long rpitch, rfs;
     int metric, ref_exact;  // ref_exact: refp holds the exact output (else the approximation)
     double* part;
+    // optional peer halos (row stripes, §8(e)): the ntop rows directly above
+    // row 0 are read from htop, the nbot rows below row h-1 from hbot (pitch
+    // hpitch) -- device pointers that may map a neighbour GPU's stripe over
+    // NVLink (CUDA IPC), so the halo exchange happens inside this kernel
+    const float* htop;
+    const float* hbot;
+    int ntop, nbot;
+    long long hpitch;
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -197,8 +205,22 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
 
         // valid staged rows / columns of this tile
         const int drow0 = y0 + A.row_off - HY;
-        const int rlo = max(0, -drow0);
-        const int rhi = min(SH - 1, A.rows_valid - 1 - drow0);
+        const int rlo = max(0, -drow0 - A.ntop);
+        const int rhi = min(SH - 1, A.rows_valid + A.nbot - 1 - drow0);
+        if (HY > 0 && (drow0 < 0 && A.ntop > 0 || drow0 + SH > A.rows_valid && A.nbot > 0)) {
+            // stripe-edge tile: the halo rows come from the peer pointers
+            // (TMA zero-filled them), columns clamped to the image
+            for (int idx = tid; idx < SH * SW; idx += kThreads) {
+                const int r = idx / SW, c = idx - r * SW;
+                const int dr = drow0 + r;
+                const float* src = nullptr;
+                if (dr < 0 && dr >= -A.ntop) src = A.htop + (long long)(A.ntop + dr) * A.hpitch;
+                else if (dr >= A.rows_valid && dr < A.rows_valid + A.nbot)
+                    src = A.hbot + (long long)(dr - A.rows_valid) * A.hpitch;
+                if (src) S[r * SW + c] = src[min(max(x0 - HXP + c, 0), A.w - 1)];
+            }
+            __syncthreads();
+        }
         const int clo = max(0, HXP - x0);
         const int chi = min(SW - 1, A.w - 1 - x0 + HXP);
         if (clo > 0 || chi < SW - 1) {  // border columns: replicate the edge (clamp)

@@ -190,6 +190,63 @@ def hotspot_stripes(bufs, power: torch.Tensor, s: Stripe, params, scheme, reach:
     return cur
 
 
+class PeerStripe:
+    """A row stripe whose neighbours' boundary rows are read inside the
+    stencil kernel through CUDA IPC mappings of their buffers (NVLink P2P on
+    one node) -- the halo exchange without a separate collective (§8(e)).
+
+    Every rank allocates its owned rows `buf` ([rows, w], device), exports it,
+    and opens the handles of ranks k-1 and k+1 (handles travel once through
+    torch.distributed's object collectives).  After the ranks have written
+    their inputs, one barrier orders those writes before the reads;
+    `stencil()` then needs no communication at all."""
+
+    def __init__(self, s: Stripe, w: int, device, group=None):
+        from . import paraprox as P
+        self.P = P
+        self.s = s
+        self.w = w
+        self.buf = torch.empty((s.rows, w), dtype=torch.float32, device=device)
+        handle, off = P.ipc_export(self.buf)
+        world = dist.get_world_size(group)
+        rank = dist.get_rank(group)
+        infos = [None] * world
+        dist.all_gather_object(infos, (handle, off, s.rows, self.buf.stride(0)), group=group)
+        self._opened = []
+        self.top = self.bot = None
+        self.top_rows = self.bot_rows = 0
+        self.top_pitch = self.bot_pitch = w
+        if rank > 0:
+            h, o, rows, pitch = infos[rank - 1]
+            base = P.ipc_open(h)
+            self._opened.append(base)
+            self.top, self.top_rows, self.top_pitch = base + o, rows, pitch
+        if rank < world - 1:
+            h, o, rows, pitch = infos[rank + 1]
+            base = P.ipc_open(h)
+            self._opened.append(base)
+            self.bot, self.bot_rows, self.bot_pitch = base + o, rows, pitch
+        if self.top_pitch != self.bot_pitch and self.top is not None and self.bot is not None:
+            raise ValueError("neighbour pitches differ")
+        self.group = group
+
+    def ready(self):
+        """Order every rank's writes of its `buf` before the peers' reads."""
+        torch.cuda.synchronize()
+        dist.barrier(group=self.group)
+
+    def stencil(self, f, scheme, reach: int, out: torch.Tensor):
+        pitch = self.top_pitch if self.top is not None else self.bot_pitch
+        return self.P.stencil_peer(self.buf, f, scheme, reach, out=out, top=self.top, top_rows=self.top_rows,
+                                   bot=self.bot, bot_rows=self.bot_rows, src_pitch=pitch)
+
+    def close(self):
+        torch.cuda.synchronize()
+        for base in self._opened:
+            self.P.ipc_close(base)
+        self._opened = []
+
+
 def _allreduce_np(a: np.ndarray, device, group=None) -> np.ndarray:
     t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).to(device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)

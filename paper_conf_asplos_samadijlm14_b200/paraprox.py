@@ -62,6 +62,10 @@ _SIGS = {
     "paraprox_stencil_lattice": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_stencil_skip_xy": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P],
     "paraprox_hotspot": [C.POINTER(HotspotParams), C.c_int, C.c_int, _P, _P, _P, _IMG, C.c_int, _P],
+    "paraprox_stencil_peer": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P, C.c_int, _P, C.c_int, C.c_longlong, _P],
+    "paraprox_ipc_export": [_P, _P, C.POINTER(C.c_longlong)],
+    "paraprox_ipc_open": [_P, C.POINTER(_P)],
+    "paraprox_ipc_close": [_P],
     "paraprox_tune_ex": [_P, C.c_int, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
     "paraprox_tune_candidates_ex": [_P, C.c_int, C.c_int, _I, _I, _I],
     "paraprox_tune_partials_ex": [_P, C.c_int, _P, _IMG, C.c_int, _D, _P],
@@ -596,3 +600,40 @@ def hotspot(temp, power, params, scheme="exact", reach: int = 0, iterations: int
     _check(_lib.paraprox_hotspot(C.byref(prm), _scheme(scheme), int(reach), _dp(temp, halo_top), _dp(power), _dp(out),
                                  C.byref(img), int(iterations), _stream(stream)), "hotspot")
     return out
+
+
+def stencil_peer(x, f: Filter, scheme, reach: int, out=None, *, top=None, top_rows: int = 0, bot=None,
+                 bot_rows: int = 0, src_pitch: int = 0, stream=None):
+    """A row stripe whose halo rows are read inside the kernel from device
+    pointers (ints) `top` (the top_rows rows right above row 0) and `bot`
+    (the bot_rows rows right below the last row), e.g. CUDA-IPC mappings of
+    the neighbours' stripes (dist.PeerStripe)."""
+    _need_cuda(x)
+    img = image_of(x)
+    out = _out_like(x, 0, 0, out)
+    _need_cuda(out)
+    _check_out(out, img)
+    _check(_lib.paraprox_stencil_peer(f.handle, _scheme(scheme), int(reach), _dp(x), _dp(out), C.byref(img),
+                                      C.c_void_p(top or 0), int(top_rows), C.c_void_p(bot or 0), int(bot_rows),
+                                      int(src_pitch), _stream(stream)), "stencil_peer")
+    return out
+
+
+def ipc_export(t: torch.Tensor):
+    """(64-byte handle, byte offset) of the CUDA allocation holding t."""
+    _need_cuda(t)
+    h = (C.c_char * 64)()
+    off = C.c_longlong()
+    _check(_lib.paraprox_ipc_export(C.c_void_p(t.data_ptr()), h, C.byref(off)), "ipc_export")
+    return bytes(h), off.value
+
+
+def ipc_open(handle: bytes) -> int:
+    buf = (C.c_char * 64).from_buffer_copy(handle)
+    p = _P()
+    _check(_lib.paraprox_ipc_open(buf, C.byref(p)), "ipc_open")
+    return p.value
+
+
+def ipc_close(base: int):
+    _check(_lib.paraprox_ipc_close(C.c_void_p(base)), "ipc_close")
