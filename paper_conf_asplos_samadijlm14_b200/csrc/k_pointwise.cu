@@ -5,7 +5,7 @@
 // PAPER.md L1158-1162 Fig. 6a): the folded filter is one tap w' = sum of all
 // weights, so the stencil degenerates to the map out = w' * in -- no halo, no
 // neighbour, nothing to stage.  This kernel streams it at copy speed: each
-// thread keeps kPU independent 128-bit loads in flight (evict-first), grid =
+// thread keeps kPU = 8 independent 128-bit loads in flight (evict-first), grid =
 // resident threads, 128-bit streaming stores.  8 B of HBM per pixel.
 //
 // Rounding matches the tile kernels bit for bit: dense fmaf(w, x, 0);
@@ -16,7 +16,23 @@
 
 namespace ppx {
 
-constexpr int kPU = 4;
+#ifndef PPX_PU
+#define PPX_PU 8
+#endif
+constexpr int kPU = PPX_PU;
+
+// streaming 128-bit load: evict-first, or with a 256-byte L2 prefetch hint
+__device__ __forceinline__ float4 ld_stream(const float4* p) {
+#if PPX_MAP_L2PF
+    float4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0, %1, %2, %3}, [%4];"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                 : "l"(p));
+    return v;
+#else
+    return __ldcs(p);
+#endif
+}
 
 template <bool SEP>
 __device__ __forceinline__ float pw(float x, float w0, float w1) {
@@ -63,7 +79,7 @@ __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict_
         float4 v[kPU];
 #pragma unroll
         for (int u = 0; u < kPU; ++u)
-            if (i + u * stride < n4) v[u] = __ldcs(i4 + i + u * stride);
+            if (i + u * stride < n4) v[u] = ld_stream(i4 + i + u * stride);
 #pragma unroll
         for (int u = 0; u < kPU; ++u)
             if (i + u * stride < n4) {
