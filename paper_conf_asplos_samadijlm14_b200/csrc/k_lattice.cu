@@ -29,6 +29,10 @@
 
 #include "k_tiles.cuh"
 
+#ifndef PPX_LAT_MIN_BLOCKS
+#define PPX_LAT_MIN_BLOCKS 2
+#endif
+
 namespace ppx {
 
 constexpr int floor_div(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
@@ -76,7 +80,7 @@ struct LatW {
 };
 
 template <int S, int R, bool SEP>
-__global__ void __launch_bounds__(kThreads, 2) k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A,
+__global__ void __launch_bounds__(kThreads, PPX_LAT_MIN_BLOCKS) k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A,
                                                          const __grid_constant__ LatW W) {
     using G = LGeom<S, R>;
     constexpr int HX = R, HXP = G::HXP, SW = G::SW, AB = G::AB, RB = G::RB, TH = G::TH, MLO = G::MLO;

@@ -14,7 +14,10 @@ namespace ppx {
 // each thread keeps kQU independent 128-bit loads of E and of A in flight per
 // iteration (grid-stride, fixed grid), so the HBM pipe stays full while the
 // fp64 division chain of MRE runs.  Other layouts walk rows.
-constexpr int kQU = 4;
+#ifndef PPX_QU
+#define PPX_QU 4
+#endif
+constexpr int kQU = PPX_QU;
 
 template <int M>
 __global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
