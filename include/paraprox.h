@@ -213,6 +213,27 @@ PARAPROX_API paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm
                                  int reach, const float* d_temp, const float* d_power, float* d_out,
                                  const paraprox_image* img, int iterations, paraprox_stream s);
 
+/* One HotSpot pass of `steps` (1..8) steps of a row stripe (img: n == 1, no
+ * halos) whose neighbours' rows are read inside the blocked kernel from peer
+ * pointers: the top_rows rows of temperature and power directly above row 0,
+ * the bot_rows rows below row h-1 (pitch src_pitch; 0 rows = the image edge).
+ * A pass needs steps x h_y rows from each peer (h_y = 1 for the exact and
+ * column schemes, 0 for row and centre).  The caller orders the passes across
+ * GPUs (paraprox_flag_wait / _set).  Asynchronous on s. */
+PARAPROX_API paraprox_status paraprox_hotspot_peer(const paraprox_hotspot_params* prm, paraprox_scheme scheme,
+                                      int reach, const float* d_temp, const float* d_power, float* d_out,
+                                      const paraprox_image* img, int steps, const float* d_top_temp,
+                                      const float* d_top_power, int top_rows, const float* d_bot_temp,
+                                      const float* d_bot_power, int bot_rows, long long src_pitch,
+                                      paraprox_stream s);
+
+/* Device-side ordering across GPUs (the flag may be a peer GPU's memory
+ * mapped by paraprox_ipc_open): wait enqueues a kernel that spins (acquire,
+ * system scope) until *d_flag >= target; set enqueues a release store of
+ * value after the preceding work of s.  Asynchronous on s. */
+PARAPROX_API paraprox_status paraprox_flag_wait(const long long* d_flag, long long target, paraprox_stream s);
+PARAPROX_API paraprox_status paraprox_flag_set(long long* d_flag, long long value, paraprox_stream s);
+
 /* ---- output quality (syncs s) ------------------------------------------ */
 
 /* Quality of d_approx against d_exact over all n*h*w elements (pooled over

@@ -639,6 +639,77 @@ paraprox_status paraprox_ipc_close(void* d_base) {
     return PARAPROX_OK;
 }
 
+paraprox_status paraprox_hotspot_peer(const paraprox_hotspot_params* prm, paraprox_scheme scheme, int reach,
+                                      const float* d_temp, const float* d_power, float* d_out,
+                                      const paraprox_image* img, int steps, const float* d_top_temp,
+                                      const float* d_top_power, int top_rows, const float* d_bot_temp,
+                                      const float* d_bot_power, int bot_rows, long long src_pitch,
+                                      paraprox_stream s) {
+    if (!prm || !d_temp || !d_power || !d_out || !img) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    if (scheme < PARAPROX_EXACT || scheme > PARAPROX_CENTER) return fail(PARAPROX_ERR_INVALID_ARG, "unknown scheme");
+    if (reach < 0 || steps < 1 || steps > kHotspotMaxSteps || top_rows < 0 || bot_rows < 0)
+        return fail(PARAPROX_ERR_INVALID_ARG, "reach, steps (1..8) or rows out of range");
+    if ((top_rows && (!d_top_temp || !d_top_power)) || (bot_rows && (!d_bot_temp || !d_bot_power)))
+        return fail(PARAPROX_ERR_INVALID_ARG, "NULL halo source");
+    paraprox_status st = check_image(img, false);
+    if (st != PARAPROX_OK) return st;
+    if (img->n != 1) return fail(PARAPROX_ERR_INVALID_ARG, "peer halos need n == 1");
+    if ((top_rows || bot_rows) && src_pitch < img->w) return fail(PARAPROX_ERR_INVALID_ARG, "src_pitch < w");
+    if (overlaps(d_temp, d_out, img) || overlaps(d_power, d_out, img))
+        return fail(PARAPROX_ERR_INVALID_ARG, "d_out overlaps an input");
+    const double c = prm->step_div_cap, gx = prm->rx_inv, gy = prm->ry_inv, gz = prm->rz_inv;
+    paraprox_filter_s f;
+    f.ky = f.kx = 3;
+    f.separable = false;
+    f.w = {0.f, (float)(c * gy), 0.f, (float)(c * gx), (float)(1.0 - 2.0 * c * gx - 2.0 * c * gy - c * gz),
+           (float)(c * gx), 0.f, (float)(c * gy), 0.f};
+    int dy, dx;
+    scheme_reaches(scheme, reach, &dy, &dx);
+    const Plan& p = get_plan(&f, dy, dx);
+    cudaStream_t cs = (cudaStream_t)s;
+    View v = view_of(img);
+    const long long ofs = (long long)img->h * img->pitch;
+    if (p.hy == 0 && p.hx == 0) {  // centre at full reach: no neighbour read, fused steps
+        Addend add;
+        add.p = d_power;
+        add.pitch = img->pitch;
+        add.fstride = ofs;
+        add.alpha = (float)c;
+        add.beta = (float)(c * gz * prm->t_amb);
+        add.steps = steps;
+        cudaError_t e = launch_stencil(p, d_temp, v, d_out, img->pitch, ofs, cs, &add);
+        if (e != cudaSuccess) return cuda_fail(e, "hotspot fused steps");
+        return PARAPROX_OK;
+    }
+    const int need = steps * p.hy;  // halo rows of `steps` steps
+    HotspotPeer peer;
+    peer.ntop = top_rows ? need : 0;
+    peer.nbot = bot_rows ? need : 0;
+    if ((top_rows && top_rows < need) || (bot_rows && bot_rows < need))
+        return fail(PARAPROX_ERR_INVALID_ARG, "fewer halo rows than steps x plan halo");
+    peer.top_t = top_rows ? d_top_temp + (long long)(top_rows - need) * src_pitch : nullptr;
+    peer.top_p = top_rows ? d_top_power + (long long)(top_rows - need) * src_pitch : nullptr;
+    peer.bot_t = d_bot_temp;
+    peer.bot_p = d_bot_power;
+    peer.pitch = src_pitch;
+    cudaError_t e = launch_hotspot_tb(p, d_temp, d_power, d_out, v, ofs, (float)c, (float)(c * gz * prm->t_amb), steps,
+                                      cs, &peer);
+    if (e != cudaSuccess) return cuda_fail(e, "hotspot peer pass");
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_flag_wait(const long long* d_flag, long long target, paraprox_stream s) {
+    if (!d_flag) return fail(PARAPROX_ERR_INVALID_ARG, "NULL flag");
+    PPX_CUDA(launch_flag_wait(d_flag, target, (cudaStream_t)s));
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_flag_set(long long* d_flag, long long value, paraprox_stream s) {
+    if (!d_flag) return fail(PARAPROX_ERR_INVALID_ARG, "NULL flag");
+    PPX_CUDA(launch_flag_set(d_flag, value, (cudaStream_t)s));
+    return PARAPROX_OK;
+}
+
 paraprox_status paraprox_quality(const float* d_exact, const float* d_approx, const paraprox_image* img,
                                  paraprox_metric m, double* h_quality, paraprox_stream s) {
     if (!h_quality) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");

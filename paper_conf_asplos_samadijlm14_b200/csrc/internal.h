@@ -101,8 +101,16 @@ cudaError_t launch_lattice(const paraprox_filter_s& f, const float* in, const Vi
 // steps of a 3x3 plan plus the power term in one pass; t, p, out share v's
 // layout (no halos)
 constexpr int kHotspotMaxSteps = 8;
+struct HotspotPeer {  // peer halo rows of a HotSpot row stripe (T and P), pitch in elements
+    const float *top_t = nullptr, *top_p = nullptr, *bot_t = nullptr, *bot_p = nullptr;
+    int ntop = 0, nbot = 0;
+    long long pitch = 0;
+};
 cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, float* out, const View& v,
-                              long long fs, float alpha, float beta, int steps, cudaStream_t s);
+                              long long fs, float alpha, float beta, int steps, cudaStream_t s,
+                              const HotspotPeer* peer = nullptr);
+cudaError_t launch_flag_wait(const long long* flag, long long target, cudaStream_t s);
+cudaError_t launch_flag_set(long long* flag, long long value, cudaStream_t s);
 // Fused stencil + quality (the tuner's candidates, the runtime's checks): the
 // plan's output is compared with `ref` (laid out like the output; ref_exact:
 // ref holds the exact output, else the approximation) instead of being

@@ -31,6 +31,12 @@ struct HsArgs {
     float w9[3][3];       // folded taps at [a + 1][b + 1] (0 where not accessed)
     float alpha, beta;
     int tiles_x, tiles_y;
+    // optional peer halos (HotSpot row stripes): the ntop rows directly above
+    // row 0 (T and P) and the nbot rows below row h-1, read from neighbour
+    // buffers (CUDA IPC / NVLink); 0 rows = the image edge (clamp)
+    const float *ptop_t, *ptop_p, *pbot_t, *pbot_p;
+    int ntop, nbot;
+    long long ppitch;
 };
 
 template <int HY, int HX>
@@ -61,17 +67,32 @@ __global__ void __launch_bounds__(HsGeom<HY, HX>::THREADS, 2) k_hotspot_tb(const
     const int oy = y0 - hy, ox = x0 - hx;  // global coordinates of staged cell (0, 0)
     const float* T = A.t + (long long)f * A.fs;
     const float* Pw = A.p + (long long)f * A.fs;
-    const bool border = oy < 0 || ox < 0 || oy + SH > A.h || ox + SW > A.w;
+    const int lo = -A.ntop, hi = A.h - 1 + A.nbot;  // valid rows (peer halo rows included)
+    const bool border = oy < lo || ox < 0 || oy + SH > hi + 1 || ox + SW > A.w;
 
-    // stage T and P over the tile + halo, clamped to the image (rows of the
-    // staged box are spread over the threads, columns over the lanes)
+    // stage T and P over the tile + halo, clamped to the valid rows and the
+    // image columns (rows of the staged box are spread over the threads,
+    // columns over the lanes); rows beyond the stripe come from the peers
     for (int r = threadIdx.x / RW; r < SH; r += G::THREADS / RW) {
         const int c = threadIdx.x % RW;
         if (c < SW) {
-            const int gy = min(max(oy + r, 0), A.h - 1), gx = min(max(ox + c, 0), A.w - 1);
-            const long long g = (long long)gy * A.pitch + gx;
-            sm[r * RW + c] = __ldg(T + g);
-            bufP[r * RW + c] = __ldg(Pw + g);
+            const int gy = min(max(oy + r, lo), hi), gx = min(max(ox + c, 0), A.w - 1);
+            const float *srcT, *srcP;
+            if (gy < 0) {
+                const long long g = (long long)(A.ntop + gy) * A.ppitch + gx;
+                srcT = A.ptop_t + g;
+                srcP = A.ptop_p + g;
+            } else if (gy >= A.h) {
+                const long long g = (long long)(gy - A.h) * A.ppitch + gx;
+                srcT = A.pbot_t + g;
+                srcP = A.pbot_p + g;
+            } else {
+                const long long g = (long long)gy * A.pitch + gx;
+                srcT = T + g;
+                srcP = Pw + g;
+            }
+            sm[r * RW + c] = *srcT;
+            bufP[r * RW + c] = *srcP;
         }
     }
     __syncthreads();
@@ -137,7 +158,7 @@ __global__ void __launch_bounds__(HsGeom<HY, HX>::THREADS, 2) k_hotspot_tb(const
             for (int idx = threadIdx.x; idx < nr * nc; idx += G::THREADS) {
                 const int r = r0 + idx / nc, cc = c0 + idx % nc;
                 const int gy = oy + r, gx = ox + cc;
-                const int cy = min(max(gy, 0), A.h - 1), cx = min(max(gx, 0), A.w - 1);
+                const int cy = min(max(gy, lo), hi), cx = min(max(gx, 0), A.w - 1);
                 if (cy != gy || cx != gx) nxt[r * RW + cc] = nxt[(cy - oy) * RW + (cx - ox)];
             }
             __syncthreads();
@@ -148,7 +169,8 @@ __global__ void __launch_bounds__(HsGeom<HY, HX>::THREADS, 2) k_hotspot_tb(const
 // taps of tap-index table order (rows, then columns ascending): the tile
 // kernels add in this order, and so does k_hotspot_tb (zeros are exact)
 cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, float* out, const View& v,
-                              long long fs, float alpha, float beta, int steps, cudaStream_t s) {
+                              long long fs, float alpha, float beta, int steps, cudaStream_t s,
+                              const HotspotPeer* peer) {
     if (steps < 1 || steps > kHsMaxS || p.separable || p.ky != 3 || p.kx != 3) return cudaErrorInvalidValue;
     for (int i = 0; i < p.ny; ++i)  // the kernel skips the corner taps: they must be zero
         for (int j = 0; j < p.nx; ++j)
@@ -167,6 +189,17 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
         for (int j = 0; j < p.nx; ++j) A.w9[p.ay[i] + 1][p.ax[j] + 1] = p.wf[i * p.nx + j];
     A.alpha = alpha;
     A.beta = beta;
+    if (peer) {
+        if (v.n != 1 || (peer->ntop && peer->ntop < steps * p.hy) || (peer->nbot && peer->nbot < steps * p.hy))
+            return cudaErrorInvalidValue;  // the halo of `steps` steps must come from the peers
+        A.ptop_t = peer->top_t;
+        A.ptop_p = peer->top_p;
+        A.pbot_t = peer->bot_t;
+        A.pbot_p = peer->bot_p;
+        A.ntop = peer->ntop;
+        A.nbot = peer->nbot;
+        A.ppitch = peer->pitch;
+    }
     A.tiles_x = (v.w + kHsTW - 1) / kHsTW;
     A.tiles_y = (v.h + kHsTH - 1) / kHsTH;
     const long long nt = (long long)A.tiles_x * A.tiles_y * v.n;
@@ -186,6 +219,40 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
     count_launch(p.hy && p.hx ? "hotspot_tb_f1_f1" : p.hy ? "hotspot_tb_f1_s0" : p.hx ? "hotspot_tb_s0_f1"
                                                                                         : "hotspot_tb_s0_s0");
     return cudaSuccess;
+}
+
+}  // namespace ppx
+
+namespace ppx {
+
+// cross-GPU step ordering for peer-halo passes: a single thread spins with
+// acquire loads (system scope: the flag may live on a peer GPU) until the
+// counter reaches `target`; the signal kernel publishes a counter with a
+// release store after everything before it in the stream
+__global__ void k_flag_wait(const volatile long long* flag, long long target) {
+    long long v;
+    for (;;) {
+        asm volatile("ld.acquire.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(flag) : "memory");
+        if (v >= target) break;
+        __nanosleep(200);
+    }
+}
+
+__global__ void k_flag_set(long long* flag, long long value) {
+    __threadfence_system();
+    asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(flag), "l"(value) : "memory");
+}
+
+cudaError_t launch_flag_wait(const long long* flag, long long target, cudaStream_t s) {
+    k_flag_wait<<<1, 1, 0, s>>>(flag, target);
+    count_launch("flag_wait");
+    return cudaGetLastError();
+}
+
+cudaError_t launch_flag_set(long long* flag, long long value, cudaStream_t s) {
+    k_flag_set<<<1, 1, 0, s>>>(flag, value);
+    count_launch("flag_set");
+    return cudaGetLastError();
 }
 
 }  // namespace ppx

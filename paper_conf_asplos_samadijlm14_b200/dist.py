@@ -247,6 +247,89 @@ class PeerStripe:
         self._opened = []
 
 
+class HotspotPeerStripes:
+    """HotSpot (NEXT-4) on row stripes with the halo exchange inside the
+    kernel: each rank keeps two temperature buffers, its power rows and a
+    pass counter in CUDA-IPC-exported memory.  A pass of up to 8 steps reads
+    the neighbours' boundary rows (8 x h_y of them) straight from their
+    buffers over NVLink, after a device-side wait for their previous pass
+    (paraprox_flag_wait on the neighbours' counters), then publishes its own
+    counter -- no host synchronisation and no collective between passes.
+    The ordering rule: before pass q every rank waits until its neighbours
+    have finished pass q - 1, which both makes their rows ready and keeps
+    them from overwriting rows still being read."""
+
+    def __init__(self, s: Stripe, w: int, device, group=None):
+        from . import paraprox as P
+        self.P = P
+        self.s = s
+        self.w = w
+        self.group = group
+        self.T = [torch.empty((s.rows, w), dtype=torch.float32, device=device) for _ in range(2)]
+        self.Pw = torch.empty((s.rows, w), dtype=torch.float32, device=device)
+        self.flag = torch.zeros(2, dtype=torch.int64, device=device)
+        mine = [P.ipc_export(t) for t in (self.T[0], self.T[1], self.Pw, self.flag)]
+        world = dist.get_world_size(group)
+        rank = dist.get_rank(group)
+        infos = [None] * world
+        dist.all_gather_object(infos, (mine, s.rows, self.T[0].stride(0)), group=group)
+        self._opened = []
+        self.nb = {}
+        for side, peer in (("top", rank - 1), ("bot", rank + 1)):
+            if 0 <= peer < world:
+                handles, rows, pitch = infos[peer]
+                ptrs = []
+                for h, off in handles:
+                    base = P.ipc_open(h)
+                    self._opened.append(base)
+                    ptrs.append(base + off)
+                self.nb[side] = dict(T=ptrs[:2], P=ptrs[2], flag=ptrs[3], rows=rows, pitch=pitch)
+        self.passes = 0
+
+    def load(self, temp_rows: torch.Tensor, power_rows: torch.Tensor):
+        """Owned rows of the initial temperature and the power; then every
+        rank's writes are ordered before the peers' reads."""
+        self.T[0].copy_(temp_rows)
+        self.Pw.copy_(power_rows)
+        self.flag.zero_()
+        self.passes = 0
+        torch.cuda.synchronize()
+        dist.barrier(group=self.group)
+
+    def run(self, params, scheme, reach: int, iterations: int):
+        """`iterations` steps; returns the buffer holding the result."""
+        P = self.P
+        left = iterations
+        while left > 0:
+            steps = min(8, left)
+            q = self.passes
+            for nb in self.nb.values():
+                P.flag_wait(nb["flag"], q)
+            kw = {}
+            pitch = self.w
+            if "top" in self.nb:
+                t = self.nb["top"]
+                kw.update(top_t=t["T"][q % 2], top_p=t["P"], top_rows=t["rows"])
+                pitch = t["pitch"]
+            if "bot" in self.nb:
+                b = self.nb["bot"]
+                kw.update(bot_t=b["T"][q % 2], bot_p=b["P"], bot_rows=b["rows"])
+                pitch = b["pitch"]
+            P.hotspot_peer(self.T[q % 2], self.Pw, params, scheme, reach, steps, self.T[(q + 1) % 2],
+                           src_pitch=pitch, **kw)
+            P.flag_set(self.flag.data_ptr(), q + 1)
+            self.passes += 1
+            left -= steps
+        return self.T[self.passes % 2]
+
+    def close(self):
+        torch.cuda.synchronize()
+        dist.barrier(group=self.group)
+        for base in self._opened:
+            self.P.ipc_close(base)
+        self._opened = []
+
+
 def _allreduce_np(a: np.ndarray, device, group=None) -> np.ndarray:
     t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).to(device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)

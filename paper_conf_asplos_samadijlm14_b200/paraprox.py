@@ -64,6 +64,10 @@ _SIGS = {
     "paraprox_hotspot": [C.POINTER(HotspotParams), C.c_int, C.c_int, _P, _P, _P, _IMG, C.c_int, _P],
     "paraprox_stencil_peer": [_P, C.c_int, C.c_int, _P, _P, _IMG, _P, C.c_int, _P, C.c_int, C.c_longlong, _P],
     "paraprox_ipc_export": [_P, _P, C.POINTER(C.c_longlong)],
+    "paraprox_hotspot_peer": [C.POINTER(HotspotParams), C.c_int, C.c_int, _P, _P, _P, _IMG, C.c_int, _P, _P, C.c_int,
+                              _P, _P, C.c_int, C.c_longlong, _P],
+    "paraprox_flag_wait": [_P, C.c_longlong, _P],
+    "paraprox_flag_set": [_P, C.c_longlong, _P],
     "paraprox_ipc_open": [_P, C.POINTER(_P)],
     "paraprox_ipc_close": [_P],
     "paraprox_tune_ex": [_P, C.c_int, _P, _IMG, C.c_double, C.c_int, _I, _I, _D, _P],
@@ -637,3 +641,28 @@ def ipc_open(handle: bytes) -> int:
 
 def ipc_close(base: int):
     _check(_lib.paraprox_ipc_close(C.c_void_p(base)), "ipc_close")
+
+
+def hotspot_peer(temp, power, params, scheme, reach: int, steps: int, out, *, top_t=None, top_p=None,
+                 top_rows: int = 0, bot_t=None, bot_p=None, bot_rows: int = 0, src_pitch: int = 0, stream=None):
+    """One HotSpot pass (<= 8 steps) of a row stripe reading its neighbours'
+    rows (device pointers as ints) inside the blocked kernel."""
+    _need_cuda(temp, power, out)
+    img = image_of(temp)
+    _check_out(out, img)
+    _check_out(power, img)
+    prm = HotspotParams(float(params["c"]), float(params["gx"]), float(params["gy"]), float(params["gz"]),
+                        float(params["tamb"]))
+    _check(_lib.paraprox_hotspot_peer(C.byref(prm), _scheme(scheme), int(reach), _dp(temp), _dp(power), _dp(out),
+                                      C.byref(img), int(steps), C.c_void_p(top_t or 0), C.c_void_p(top_p or 0),
+                                      int(top_rows), C.c_void_p(bot_t or 0), C.c_void_p(bot_p or 0), int(bot_rows),
+                                      int(src_pitch), _stream(stream)), "hotspot_peer")
+    return out
+
+
+def flag_wait(flag_ptr: int, target: int, *, stream=None):
+    _check(_lib.paraprox_flag_wait(C.c_void_p(flag_ptr), int(target), _stream(stream)), "flag_wait")
+
+
+def flag_set(flag_ptr: int, value: int, *, stream=None):
+    _check(_lib.paraprox_flag_set(C.c_void_p(flag_ptr), int(value), _stream(stream)), "flag_set")

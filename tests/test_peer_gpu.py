@@ -105,3 +105,53 @@ def test_peer_stripes_ipc_two_processes(world):
         p.join(timeout=60)
     for r in range(world):
         assert res[r] == "ok", res[r]
+
+
+def _hotspot_worker(rank, world, port, q):
+    try:
+        import sys
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        import paper_conf_asplos_samadijlm14_b200 as pkg
+        from paper_conf_asplos_samadijlm14_b200 import dist as D
+        from workloads import hotspot as H
+        P = pkg.paraprox
+        h, w = 150, 260
+        t, p = H.frames(1, h, w, 3)
+        td, pd = torch.from_numpy(t[0]).cuda(), torch.from_numpy(p[0]).cuda()
+        s = D.stripe_of(h, world, rank, cap=8)
+        hs = D.HotspotPeerStripes(s, w, "cuda")
+        for scheme, reach in (("exact", 0), ("col", 1), ("row", 1), ("center", 1)):
+            for iters in (1, 8, 19):
+                hs.load(td[s.r0:s.r1], pd[s.r0:s.r1])
+                got = hs.run(H.PARAMS, scheme, reach, iters)
+                full = P.hotspot(td, pd, H.PARAMS, scheme, reach, iters)
+                torch.cuda.synchronize()
+                assert torch.equal(got, full[s.r0:s.r1]), (rank, scheme, iters, float((got - full[s.r0:s.r1]).abs().max()))
+        hs.close()
+        q.put((rank, "ok"))
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, traceback.format_exc()))
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_hotspot_peer_stripes_ipc(world):
+    """HotSpot passes of a striped grid with in-kernel peer halos and
+    device-side pass ordering: bit-identical to the whole grid."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_hotspot_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=600) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(world):
+        assert res[r] == "ok", res[r]
