@@ -42,8 +42,14 @@
 namespace ppx {
 
 constexpr int kTW = 128;                 // tile width (outputs)
-constexpr int kRB = 8;                   // output rows per thread
-constexpr int kWarps = 8;                // 256 threads
+#ifndef PPX_KRB
+#define PPX_KRB 8
+#endif
+#ifndef PPX_KWARPS
+#define PPX_KWARPS 8
+#endif
+constexpr int kRB = PPX_KRB;             // output rows per thread
+constexpr int kWarps = PPX_KWARPS;       // 256 threads
 constexpr int kTH = kRB * kWarps;        // 64 tile rows
 constexpr int kThreads = 32 * kWarps;
 
