@@ -18,3 +18,9 @@ timeout 900 python tools/toq_sweep.py > gpurun_out/toq_sweep.log 2>&1; echo swee
 timeout 400 python tools/kbench.py > gpurun_out/kbench.jsonl 2>&1; echo kbench rc=$?
 timeout 600 python tools/convsep.py > gpurun_out/convsep.log 2>&1; echo convsep rc=$?
 timeout 600 python tools/hotspot.py > gpurun_out/hotspot.log 2>&1; echo hotspot rc=$?
+if [ -z "$NO_NCU" ]; then
+for c in c1 c3 c4; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_tiles|k_pointwise|k_lattice" -c 4 -o gpurun_out/prof_$c -f python tools/prof_run.py --workload $c --schemes exact:0,center:9 --reps 1 > gpurun_out/ncu_$c.log 2>&1; echo ncu $c rc=$?
+done
+fi
+bash tools/sanitize.sh
