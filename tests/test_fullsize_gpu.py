@@ -97,3 +97,49 @@ def test_c1_gauss3_512_batch(P, O):
         g = P.stencil_approx(xd, f, s, d).cpu().numpy()
         o = O.stencil_approx(x, w, s, d)
         assert np.all(np.abs(g - o) <= RTOL * np.abs(o)), (s, d)
+
+
+def test_c4_lattice_sampled(P, O):
+    """NEXT-1 at c4's size: the row lattice (reach 1 and 4) on 32768^2, sampled
+    patches against the exact stencil on the rebuilt array X~ (oracle lattice
+    map + oracle exact stencil on crops with a radius margin)."""
+    w = F.conv(9)
+    f = P.Filter(w)
+    h = wd = 32768
+    x = W.periodic(h, wd, tile=4096, seed=0)
+    xd = torch.from_numpy(x).cuda()
+    size, r = 48, 4
+    for d in (1, 4):
+        g = P.stencil_lattice(xd, f, "row", d).cpu().numpy()
+        assert P.last_kernel().startswith("lattice_dense"), P.last_kernel()
+        gy = O.lattice_map(h, d)
+        for (y0, x0) in patches(h, wd, size):
+            cy0, cx0 = max(0, y0 - r), max(0, x0 - r)
+            cy1, cx1 = min(h, y0 + size + r), min(wd, x0 + size + r)
+            xt = x[gy[cy0:cy1]][:, cx0:cx1]  # rows replaced by their accessed rows
+            o = O.stencil_exact(xt, w)
+            b = RTOL * O.stencil_exact(np.abs(xt), np.abs(w))
+            sl = (slice(y0 - cy0, y0 - cy0 + size), slice(x0 - cx0, x0 - cx0 + size))
+            assert np.all(np.abs(g[y0:y0 + size, x0:x0 + size] - o[sl]) <= b[sl]), (d, y0, x0)
+        del g
+    del xd
+    torch.cuda.empty_cache()
+
+
+def test_c3_lattice_sampled_frames(P, O):
+    wy, wx = F.separable(7)
+    f = P.Filter(wy=wy, wx=wx)
+    base = W.frames(2, 2160, 3840, 30)
+    xd = torch.empty((256, 2160, 3840), device="cuda")
+    for k in range(256):
+        xd[k].copy_(torch.from_numpy(base[k % 2]))
+    for d in (1, 4):
+        out = P.stencil_lattice(xd, f, "row", d)
+        for k in (0, 255):
+            g = out[k].cpu().numpy()
+            o = O.stencil_lattice_xy(base[k % 2], (wy, wx), d, 0)
+            b = RTOL * O.stencil_lattice_xy(base[k % 2], (np.abs(wy), np.abs(wx)), d, 0)
+            assert np.all(np.abs(g - o) <= b), (d, k)
+        del out
+    del xd
+    torch.cuda.empty_cache()
