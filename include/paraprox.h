@@ -359,6 +359,16 @@ PARAPROX_API paraprox_status paraprox_runtime_sync(paraprox_runtime rt);
 PARAPROX_API paraprox_status paraprox_runtime_state(paraprox_runtime rt, paraprox_scheme* scheme, int* reach,
                                        long long* invocations, long long* checks, long long* backoffs,
                                        double* last_quality);
+/* Profiled training (call before _train; the paper's runtime "profiles the
+ * kernels and picks ... the best performance"): every candidate
+ * that meets the TOQ on the training frames, and the exact stencil, is timed
+ * there (CUDA events, best of 3); rung 0 is the fastest passing candidate and
+ * the ladder continues with the passing candidates of strictly higher
+ * training quality, then EXACT.  Not bit-reproducible across runs (timings). */
+PARAPROX_API paraprox_status paraprox_runtime_set_profiled(paraprox_runtime rt, int enable);
+/* Measured ms per candidate in tuner order, then the exact stencil (NaN where
+ * not measured); *n = candidates + 1. */
+PARAPROX_API paraprox_status paraprox_runtime_timings(paraprox_runtime rt, int cap, int* n, double* ms);
 /* The ladder: *n rungs, at most cap written (arrays may be NULL). */
 PARAPROX_API paraprox_status paraprox_runtime_ladder(paraprox_runtime rt, int cap, int* n,
                                         paraprox_scheme* schemes, int* reaches, double* train_quality);

@@ -21,6 +21,7 @@
 //     ladder.  Exact never moves.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cmath>
 #include <mutex>
 #include <new>
@@ -40,6 +41,9 @@ struct paraprox_runtime_s {
     long long invocations = 0, checks = 0, backoffs = 0;
     double last_q = 0.0;
     bool trained = false;
+    bool profiled = false;       // R1': pick the fastest passing candidate by measurement
+    std::vector<double> time_ms;  // per candidate (profiled mode; NaN = not measured), then exact
+
     // check state
     float* d_exact = nullptr;
     size_t exact_cap = 0;
@@ -130,20 +134,83 @@ paraprox_status paraprox_runtime_train(paraprox_runtime rt, const float* d_train
     for (size_t k = 0; k < c.size(); ++k) rt->train_q[k] = quality_of(parts.data() + 3 * k, rt->m);
     // R1 / R2
     rt->ladder.clear();
+    rt->time_ms.assign(c.size() + 1, NAN);
     int first = -1;
-    for (size_t k = 0; k < c.size(); ++k)
-        if (rt->train_q[k] >= rt->toq) {
-            first = (int)k;
-            break;
-        }
-    if (first >= 0) {
-        rt->ladder.push_back(first);
-        double best = rt->train_q[first];
-        for (size_t k = first + 1; k < c.size(); ++k)
-            if (rt->train_q[k] > best) {
-                rt->ladder.push_back((int)k);
-                best = rt->train_q[k];
+    if (!rt->profiled) {
+        for (size_t k = 0; k < c.size(); ++k)
+            if (rt->train_q[k] >= rt->toq) {
+                first = (int)k;
+                break;
             }
+        if (first >= 0) {
+            rt->ladder.push_back(first);
+            double best = rt->train_q[first];
+            for (size_t k = first + 1; k < c.size(); ++k)
+                if (rt->train_q[k] > best) {
+                    rt->ladder.push_back((int)k);
+                    best = rt->train_q[k];
+                }
+        }
+    } else {
+        // R1' ("profiles the kernels and picks ... the best
+        // performance"): every passing candidate and the exact stencil are
+        // timed on the training frames (CUDA events, best of 3 after a warm-up
+        // launch); rung 0 is the fastest passing one, the ladder continues
+        // with the passing candidates of strictly higher training quality in
+        // increasing quality, then EXACT
+        cudaStream_t cs = (cudaStream_t)s;
+        // timing output with the training image's layout (run_stencil shares it)
+        const long long fs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
+        const long long need = (long long)(img->n - 1) * fs + (long long)(img->h - 1) * img->pitch + img->w;
+        void* tmp = nullptr;
+        PPX_CUDA(scratch_alloc(&tmp, sizeof(float) * need, cs));
+        cudaEvent_t e0, e1;
+        PPX_CUDA(cudaEventCreate(&e0));
+        PPX_CUDA(cudaEventCreate(&e1));
+        auto time_it = [&](int dy, int dx, double* ms) -> paraprox_status {
+            float best = INFINITY;
+            for (int rep = 0; rep < 4; ++rep) {
+                PPX_CUDA(cudaEventRecord(e0, cs));
+                paraprox_status st2 = run_stencil(rt->f, dy, dx, d_train, (float*)tmp, img, s);
+                if (st2 != PARAPROX_OK) return st2;
+                PPX_CUDA(cudaEventRecord(e1, cs));
+                PPX_CUDA(cudaEventSynchronize(e1));
+                float t = 0.f;
+                PPX_CUDA(cudaEventElapsedTime(&t, e0, e1));
+                if (rep > 0 && t < best) best = t;
+            }
+            *ms = best;
+            return PARAPROX_OK;
+        };
+        paraprox_status st2 = PARAPROX_OK;
+        double best_ms = INFINITY;
+        for (size_t k = 0; k < c.size() && st2 == PARAPROX_OK; ++k) {
+            if (rt->train_q[k] < rt->toq) continue;
+            st2 = time_it(c[k].dy, c[k].dx, &rt->time_ms[k]);
+            if (st2 == PARAPROX_OK && rt->time_ms[k] < best_ms) {
+                best_ms = rt->time_ms[k];
+                first = (int)k;
+            }
+        }
+        if (st2 == PARAPROX_OK) st2 = time_it(0, 0, &rt->time_ms[c.size()]);
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        cudaFreeAsync(tmp, cs);
+        if (st2 != PARAPROX_OK) return st2;
+        if (first >= 0) {
+            std::vector<int> up;
+            for (size_t k = 0; k < c.size(); ++k)
+                if ((int)k != first && rt->train_q[k] >= rt->toq && rt->train_q[k] > rt->train_q[first])
+                    up.push_back((int)k);
+            std::stable_sort(up.begin(), up.end(), [&](int a, int b) { return rt->train_q[a] < rt->train_q[b]; });
+            rt->ladder.push_back(first);
+            double best = rt->train_q[first];
+            for (int k : up)
+                if (rt->train_q[k] > best) {
+                    rt->ladder.push_back(k);
+                    best = rt->train_q[k];
+                }
+        }
     }
     rt->ladder.push_back(-1);
     rt->rung = 0;
@@ -270,6 +337,23 @@ paraprox_status paraprox_runtime_state(paraprox_runtime rt, paraprox_scheme* sch
     if (checks) *checks = rt->checks;
     if (backoffs) *backoffs = rt->backoffs;
     if (last_quality) *last_quality = rt->last_q;
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_runtime_set_profiled(paraprox_runtime rt, int enable) {
+    if (!rt) return fail(PARAPROX_ERR_INVALID_ARG, "runtime is NULL");
+    std::lock_guard<std::mutex> lk(rt->mu);
+    rt->profiled = enable != 0;
+    return PARAPROX_OK;
+}
+
+paraprox_status paraprox_runtime_timings(paraprox_runtime rt, int cap, int* n, double* ms) {
+    if (!rt || !n) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
+    std::lock_guard<std::mutex> lk(rt->mu);
+    if (!rt->trained) return fail(PARAPROX_ERR_INVALID_ARG, "runtime not trained");
+    *n = (int)rt->time_ms.size();
+    for (int i = 0; i < *n && i < cap; ++i)
+        if (ms) ms[i] = rt->time_ms[i];
     return PARAPROX_OK;
 }
 

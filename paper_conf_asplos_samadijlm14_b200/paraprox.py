@@ -85,6 +85,8 @@ _SIGS = {
     "paraprox_runtime_state": [_P, _I, _I, C.POINTER(C.c_longlong), C.POINTER(C.c_longlong),
                                C.POINTER(C.c_longlong), _D],
     "paraprox_runtime_ladder": [_P, C.c_int, _I, _I, _I, _D],
+    "paraprox_runtime_set_profiled": [_P, C.c_int],
+    "paraprox_runtime_timings": [_P, C.c_int, _I, _D],
     "paraprox_quality": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials": [_P, _P, _IMG, C.c_int, _D, _P],
     "paraprox_quality_partials_async": [_P, _P, _IMG, C.c_int, _P, _P],
@@ -493,12 +495,22 @@ class Runtime:
     stencil on the device and a quality below ``toq`` moves one rung down the
     ladder."""
 
-    def __init__(self, f: Filter, toq: float, metric="mre", check_every: int = 40):
+    def __init__(self, f: Filter, toq: float, metric="mre", check_every: int = 40, profiled: bool = False):
         self._f = f
         h = _P()
         _check(_lib.paraprox_runtime_create(f.handle, float(toq), _metric(metric), int(check_every), C.byref(h)),
                "runtime_create")
         self._h = h
+        if profiled:
+            _check(_lib.paraprox_runtime_set_profiled(h, 1), "runtime_set_profiled")
+
+    def timings(self):
+        """Measured ms per candidate (tuner order), then exact; NaN = not timed."""
+        n = C.c_int()
+        _check(_lib.paraprox_runtime_timings(self._h, 0, C.byref(n), None), "runtime_timings")
+        ms = (C.c_double * max(1, n.value))()
+        _check(_lib.paraprox_runtime_timings(self._h, n.value, C.byref(n), ms), "runtime_timings")
+        return [ms[i] for i in range(n.value)]
 
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:

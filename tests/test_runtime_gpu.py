@@ -123,3 +123,30 @@ def test_check_overhead_at_one_in_forty(P):
     chk = min(c for _, c in runs)
     print(f"runtime overhead at 1/40 checks: {100 * (chk / base - 1):.2f} %  ({base:.3f} ms -> {chk:.3f} ms)")
     assert chk / base < 1.15
+
+
+def test_profiled_training_picks_the_fastest_passing(P):
+    """R1': with profiling on, rung 0 is the fastest candidate
+    that meets the TOQ on the training frames, by the runtime's own timings;
+    the ladder then rises in training quality and ends at exact."""
+    f = P.Filter(F.conv(9))
+    train = dev(W.frames(2, 1024, 1024, 0))
+    rt = P.Runtime(f, 0.9, "l2", check_every=10, profiled=True)
+    st = rt.train(train)
+    lad = rt.ladder()
+    ms = rt.timings()
+    cands = P.tune_candidates(f)
+    assert len(ms) == len(cands) + 1 and not np.isnan(ms[-1])
+    parts = P.tune_partials(train, f, "l2")
+    qs = [P.quality_from_partials(parts[3 * k:3 * k + 3], "l2") for k in range(len(cands))]
+    passing = [k for k, q in enumerate(qs) if q >= 0.9]
+    assert passing, qs
+    fastest = min(passing, key=lambda k: ms[k])
+    assert (st["scheme"], st["reach"]) == cands[fastest]
+    assert all(not np.isnan(ms[k]) for k in passing)
+    tq = [q for _, _, q in lad]
+    assert all(a < b for a, b in zip(tq, tq[1:])) and lad[-1][:2] == ("exact", 0)
+    x = dev(W.frames(1, 1024, 1024, 50))
+    out = torch.empty_like(x)
+    rt.run(x, out=out)
+    assert torch.equal(out, P.stencil_approx(x, f, st["scheme"], st["reach"]))
