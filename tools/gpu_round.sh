@@ -24,3 +24,13 @@ for c in c1 c3 c4; do
 done
 fi
 bash tools/sanitize.sh
+# summarise the ncu captures here on the box (gpurun_out/ must stay < 64 MiB)
+for c in c1 c2 c3 c4; do
+  if [ -f gpurun_out/prof_$c.ncu-rep ]; then
+    python tools/ncu_summary.py full gpurun_out/prof_$c.ncu-rep --workload $c --traffic gpurun_out/traffic_box.json > gpurun_out/ncu_full_$c.md 2>/dev/null
+    rm -f gpurun_out/prof_$c.ncu-rep
+  fi
+done
+python tools/ncu_summary.py launches gpurun_out/launches_c2.csv > gpurun_out/launches_c2.md 2>/dev/null
+du -sh gpurun_out
+

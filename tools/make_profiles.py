@@ -91,7 +91,21 @@ def main():
     if os.path.exists(os.path.join(OUT, "kbench.jsonl")):
         shutil.copy(os.path.join(OUT, "kbench.jsonl"), os.path.join(PROF, f"{tag}_kbench.jsonl"))
     summ = os.path.join(ROOT, "tools", "ncu_summary.py")
-    if os.path.exists(os.path.join(OUT, "launches_c2.csv")):
+    # summaries made on the GPU box (the captures themselves stay there)
+    for wl in ("c1", "c2", "c3", "c4"):
+        md = os.path.join(OUT, f"ncu_full_{wl}.md")
+        if os.path.exists(md):
+            shutil.copy(md, os.path.join(PROF, f"{tag}_ncu_full_{wl}.md"))
+    if os.path.exists(os.path.join(OUT, "launches_c2.md")):
+        shutil.copy(os.path.join(OUT, "launches_c2.md"), os.path.join(PROF, f"{tag}_launches_c2.md"))
+    box = os.path.join(OUT, "traffic_box.json")
+    if os.path.exists(box):
+        tj = os.path.join(PROF, "traffic.json")
+        d = json.load(open(tj)) if os.path.exists(tj) else {}
+        for wl, kv in json.load(open(box)).items():
+            d.setdefault(wl, {}).update(kv)
+        json.dump(d, open(tj, "w"), indent=1, sort_keys=True)
+    if os.path.exists(os.path.join(OUT, "launches_c2.csv")) and not os.path.exists(os.path.join(OUT, "launches_c2.md")):
         with open(os.path.join(PROF, f"{tag}_launches_c2.md"), "w") as fh:
             subprocess.run([sys.executable, summ, "launches", os.path.join(OUT, "launches_c2.csv")], stdout=fh, check=True)
     for wl in ("c1", "c2", "c3", "c4"):
