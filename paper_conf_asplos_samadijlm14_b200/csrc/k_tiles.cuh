@@ -152,6 +152,54 @@ __device__ __forceinline__ void static_for(F&& f) {
     static_for_impl(f, std::make_integer_sequence<int, N>{});
 }
 
+// Out-of-line epilogue of the rarely used modes: the additive input
+// (HotSpot's power: out = acc + alpha * p + beta) and/or the fused quality
+// (compare with the reference instead of storing, accumulate into racc).
+static __device__ __noinline__ void tile_epilogue_special(const float* addp, long long apitch, long long afs, float alpha,
+                                                   float beta, const float* refp, long long rpitch, long long rfs,
+                                                   int metric, int ref_exact, float* out, long long opitch,
+                                                   long long ofs, int h, int w, int f, int yb, int x,
+                                                   const float (&r)[kRB][4], RAcc& racc) {
+    for (int k = 0; k < kRB; ++k) {
+        const int y = yb + k;
+        if (y >= h || x >= w) continue;
+        float r4[4] = {r[k][0], r[k][1], r[k][2], r[k][3]};
+        if (addp) {
+            const float* ap = addp + (long long)f * afs + x + (long long)y * apitch;
+            float a4[4] = {0.f, 0.f, 0.f, 0.f};
+            if (x + 3 < w) {
+                const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
+                a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
+            } else {
+                for (int c = 0; c < 4; ++c)
+                    if (x + c < w) a4[c] = ap[c];
+            }
+            for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(alpha, a4[c], r4[c]), beta);
+        }
+        if (refp) {
+            const float* rp = refp + (long long)f * rfs + x + (long long)y * rpitch;
+            float q4[4] = {0.f, 0.f, 0.f, 0.f};
+            if (x + 3 < w) {
+                const float4 t = __ldcs(reinterpret_cast<const float4*>(rp));
+                q4[0] = t.x, q4[1] = t.y, q4[2] = t.z, q4[3] = t.w;
+            } else {
+                for (int c = 0; c < 4; ++c)
+                    if (x + c < w) q4[c] = rp[c];
+            }
+            for (int c = 0; c < 4; ++c)
+                if (x + c < w) racc.add(metric, ref_exact ? q4[c] : r4[c], ref_exact ? r4[c] : q4[c]);
+        } else {
+            float* o = out + (long long)f * ofs + (long long)y * opitch + x;
+            if (x + 3 < w) {
+                __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
+            } else {
+                for (int c = 0; c < 4; ++c)
+                    if (x + c < w) __stcs(o + c, r4[c]);
+            }
+        }
+    }
+}
+
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
 __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
                                                        const TileArgs A, const __grid_constant__ TapW W) {
@@ -315,50 +363,40 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             }
         }
 
-        // stores: 128-bit streaming where the 4 columns are inside the image
+        // stores: 128-bit streaming where the 4 columns are inside the image;
+        // the additive-input and fused-quality epilogues live out of line so
+        // the plain stencils keep a lean epilogue (and their register budget)
         const int x = x0 + 4 * lane;
-        float* obase = A.out + (long long)f * A.ofs + x;
+#ifdef PPX_NO_SPECIAL_EPI  // A/B only: the plain store epilogue
+        if (false) {
+#else
+        if (A.addp || A.refp) {
+#endif
+            float r[kRB][4];
 #pragma unroll
-        for (int k = 0; k < kRB; ++k) {
-            const int y = y0 + ty0 + k;
-            if (y < A.h && x < A.w) {
-                float* o = obase + (long long)y * A.opitch;
-                float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
-                if (A.addp) {  // additive input (HotSpot's power, single steps and stripes)
-                    const float* ap = A.addp + (long long)f * A.afs + x + (long long)y * A.apitch;
-                    float a4[4] = {0.f, 0.f, 0.f, 0.f};
+            for (int k = 0; k < kRB; ++k) {
+                r[k][0] = acc[k][0].x;
+                r[k][1] = acc[k][0].y;
+                r[k][2] = acc[k][1].x;
+                r[k][3] = acc[k][1].y;
+            }
+            tile_epilogue_special(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.refp, A.rpitch, A.rfs, A.metric,
+                                  A.ref_exact, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0, x, r, racc);
+        } else {
+            float* obase = A.out + (long long)f * A.ofs + x;
+#pragma unroll
+            for (int k = 0; k < kRB; ++k) {
+                const int y = y0 + ty0 + k;
+                if (y < A.h && x < A.w) {
+                    float* o = obase + (long long)y * A.opitch;
                     if (x + 3 < A.w) {
-                        const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
-                        a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
+                        __stcs(reinterpret_cast<float4*>(o), make_float4(acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y));
                     } else {
+                        const float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
 #pragma unroll
                         for (int c = 0; c < 4; ++c)
-                            if (x + c < A.w) a4[c] = ap[c];
+                            if (x + c < A.w) __stcs(o + c, r4[c]);
                     }
-#pragma unroll
-                    for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
-                }
-                if (A.refp) {  // fused quality: no store
-                    const float* rp = A.refp + (long long)f * A.rfs + x + (long long)y * A.rpitch;
-                    float q4[4] = {0.f, 0.f, 0.f, 0.f};
-                    if (x + 3 < A.w) {
-                        const float4 t = __ldcs(reinterpret_cast<const float4*>(rp));
-                        q4[0] = t.x, q4[1] = t.y, q4[2] = t.z, q4[3] = t.w;
-                    } else {
-#pragma unroll
-                        for (int c = 0; c < 4; ++c)
-                            if (x + c < A.w) q4[c] = rp[c];
-                    }
-#pragma unroll
-                    for (int c = 0; c < 4; ++c)
-                        if (x + c < A.w)
-                            racc.add(A.metric, A.ref_exact ? q4[c] : r4[c], A.ref_exact ? r4[c] : q4[c]);
-                } else if (x + 3 < A.w) {
-                    __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
-                } else {
-#pragma unroll
-                    for (int c = 0; c < 4; ++c)
-                        if (x + c < A.w) __stcs(o + c, r4[c]);
                 }
             }
         }
