@@ -238,19 +238,31 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
     // scheduled as soon as SMs free up.
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    // the CTA's k-th tile: strided (b + k G: concurrently running CTAs take
+    // neighbouring tiles) or, with PPX_TILE_RUNS, a contiguous run of tiles
+    // along the rows (a tile's left halo was fetched by the same CTA just before)
+#if PPX_TILE_RUNS
+    const int per = (A.ntiles + gridDim.x - 1) / gridDim.x;
+    const int t_begin = blockIdx.x * per, t_end = min(A.ntiles, t_begin + per);
+    auto tile_at = [&](int k) { return t_begin + k; };
+    auto in_range = [&](int t) { return t < t_end; };
+#else
+    auto tile_at = [&](int k) { return (int)blockIdx.x + k * (int)gridDim.x; };
+    auto in_range = [&](int t) { return t < A.ntiles; };
+#endif
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s) {
-            const int t = blockIdx.x + s * gridDim.x;
-            if (t < A.ntiles) issue(t, s);
+            const int t = tile_at(s);
+            if (in_range(t)) issue(t, s);
         }
 
     RAcc racc;  // fused-quality partials (A.refp)
     int it = 0;
-    for (int tile = blockIdx.x; tile < A.ntiles; tile += gridDim.x, ++it) {
+    for (int tile = tile_at(0); in_range(tile); tile = tile_at(++it)) {
         const int s = it % G::STAGES;
         if (tid == 0) {
-            const int ahead = tile + (G::STAGES - 1) * gridDim.x;
-            if (ahead < A.ntiles) issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+            const int ahead = tile_at(it + G::STAGES - 1);
+            if (in_range(ahead)) issue(ahead, (it + G::STAGES - 1) % G::STAGES);
         }
         int f, y0, x0;
         coords(tile, f, y0, x0);

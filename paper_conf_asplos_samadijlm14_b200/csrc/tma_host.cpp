@@ -2,6 +2,7 @@
 // point (the library does not link libcuda directly).
 #include <cudaTypedefs.h>
 
+#include <cstdlib>
 #include <mutex>
 
 #include "tma.cuh"
@@ -21,6 +22,20 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
     return fn;
 }
 
+// L2 promotion of the TMA loads; PARAPROX_TMA_L2PROMO = 0 / 64 / 128 / 256
+// overrides it (A/B only)
+static CUtensorMapL2promotion l2_promotion() {
+    static CUtensorMapL2promotion v = [] {
+        const char* e = std::getenv("PARAPROX_TMA_L2PROMO");
+        const int b = e ? std::atoi(e) : 256;
+        return b == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+               : b == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+               : b == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+                          : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }();
+    return v;
+}
+
 bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n, long long pitch,
                     long long fstride, int box_w, int box_h) {
     auto enc = get_encoder();
@@ -34,7 +49,7 @@ bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n,
     cuuint32_t box[3] = {(cuuint32_t)box_w, (cuuint32_t)box_h, 1};
     cuuint32_t estr[3] = {1, 1, 1};
     CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(base), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, l2_promotion(),
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
