@@ -92,6 +92,14 @@ bool force_generic() {
 
 }  // namespace
 
+bool tma_store_enabled() {
+    static const bool v = [] {
+        const char* e = std::getenv("PARAPROX_TMA_STORE");
+        return !(e && e[0] == '0');
+    }();
+    return v;
+}
+
 void register_tile_instance(const TileInstance& ti) {
     for (const Entry& o : reg())  // the same instance serves several radii
         if (o.ti.fn == ti.fn) return;
@@ -118,6 +126,12 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     const int box_w = kTW + 2 * round4(e.ti.hx), box_h = kTH + 2 * e.ti.hy;
     if (!encode_tmap_3d(&tmap, in + (long long)v.lo * v.pitch, v.w, rows_valid, v.n, v.pitch, fstride, box_w, box_h))
         return cudaSuccess;
+    // output map for the TMA-store epilogue (PPX_TMA_STORE); a layout it
+    // cannot describe keeps the register-store epilogue
+    CUtensorMap omap = tmap;  // (unused unless A.tma_store)
+    const bool tma_store = !qo && !add && tma_store_enabled() &&
+                           encode_tmap_3d(&omap, out, v.w, v.h, v.n, opitch, v.n > 1 ? ofs : (long long)v.h * opitch,
+                                          kTW, kTH);
     {
         std::lock_guard<std::mutex> lk(g_mu);
         if (!e.ready[dev]) {
@@ -164,6 +178,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.ntop = ph ? ph->ntop : 0;
     A.nbot = ph ? ph->nbot : 0;
     A.hpitch = ph ? ph->pitch : 0;
+    A.tma_store = tma_store ? 1 : 0;
     if (qo && ((reinterpret_cast<uintptr_t>(qo->ref) & 15) || (qo->rpitch & 3) || (v.n > 1 && (qo->rfs & 3))))
         return cudaSuccess;
     TapW W = {};
@@ -188,7 +203,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    err = cudaLaunchKernelEx(&cfg, e.ti.fn, tmap, A, W);
+    err = cudaLaunchKernelEx(&cfg, e.ti.fn, tmap, A, W, omap);
     if (err != cudaSuccess) return err;
     count_launch(qo ? "tile_quality" : e.ti.name);
     *taken = true;

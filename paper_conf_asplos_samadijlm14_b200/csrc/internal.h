@@ -154,6 +154,11 @@ paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, cons
                                    paraprox_metric m, const std::vector<Candidate>& cands, double* h_partials,
                                    paraprox_stream s);
 
+// TMA-store epilogues of the tile and lattice kernels (default on);
+// PARAPROX_TMA_STORE=0 keeps 128-bit register stores (A/B, and
+// compute-sanitizer initcheck, which does not see bulk-tensor stores)
+bool tma_store_enabled();
+
 void count_launch(const char* name);
 extern std::atomic<unsigned long long> g_launches;
 extern thread_local const char* t_last_kernel;

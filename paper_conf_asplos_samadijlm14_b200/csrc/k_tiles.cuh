@@ -83,6 +83,9 @@ struct TileArgs {
     const float* hbot;
     int ntop, nbot;
     long long hpitch;
+    // plain stencils: outputs leave as one TMA store per tile (omap) instead
+    // of 128-bit register stores (PARAPROX_TMA_STORE=0 selects the latter)
+    int tma_store;
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -94,7 +97,9 @@ struct Geom {
     static constexpr int SH = kTH + 2 * HY;    // staged rows
     static constexpr int STAGE_BYTES = SW * SH * 4;
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
-    static constexpr int STAGES = (3 * STAGE_STRIDE <= 110 * 1024 && PPX_TILE_MAX_STAGES >= 3) ? 3 : 2;
+    // as many stages as fit two CTAs per SM (<= 110 KiB each), 2..MAX
+    static constexpr int FIT = (110 * 1024) / STAGE_STRIDE;
+    static constexpr int STAGES = FIT < 2 ? 2 : (FIT < PPX_TILE_MAX_STAGES ? FIT : PPX_TILE_MAX_STAGES);
     static constexpr int SMEM = STAGES * STAGE_STRIDE;
 };
 
@@ -202,7 +207,8 @@ static __device__ __noinline__ void tile_epilogue_special(const float* addp, lon
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
 __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
-                                                       const TileArgs A, const __grid_constant__ TapW W) {
+                                                       const TileArgs A, const __grid_constant__ TapW W,
+                                                       const __grid_constant__ CUtensorMap omap) {
     using G = Geom<HY, HX>;
     constexpr int HXP = G::HXP, SW = G::SW, SH = G::SH, NV = 4 + 2 * HXP;
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -262,7 +268,11 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
         const int s = it % G::STAGES;
         if (tid == 0) {
             const int ahead = tile_at(it + G::STAGES - 1);
-            if (in_range(ahead)) issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+            if (in_range(ahead)) {
+                // the stage refilled held the previous tile's output (TMA store)
+                if (A.tma_store) bulk_wait_read_all();
+                issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+            }
         }
         int f, y0, x0;
         coords(tile, f, y0, x0);
@@ -394,6 +404,20 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             }
             tile_epilogue_special(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.refp, A.rpitch, A.rfs, A.metric,
                                   A.ref_exact, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0, x, r, racc);
+        } else if (A.tma_store) {
+            // the tile's outputs replace its consumed input stage ([kTH][kTW])
+            // and leave as one TMA store (out-of-image elements are clipped)
+            __syncthreads();  // every thread has finished reading the stage
+#pragma unroll
+            for (int k = 0; k < kRB; ++k)
+                reinterpret_cast<float4*>(S + (ty0 + k) * kTW)[lane] =
+                    make_float4(acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y);
+            fence_proxy_async();  // generic-proxy writes -> visible to the TMA unit
+            __syncthreads();
+            if (tid == 0) {
+                tma_store_3d(&omap, S, x0, y0, f);
+                bulk_commit();
+            }
         } else {
             float* obase = A.out + (long long)f * A.ofs + x;
 #pragma unroll
@@ -414,6 +438,7 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
         }
         __syncthreads();  // stage s fully consumed before it is refilled
     }
+    if (A.tma_store && tid == 0) bulk_wait_all();
     if (A.refp) {  // deterministic: fixed tile order per CTA, fixed reduction tree
         double s0, s1;
         racc.get(A.metric, s0, s1);
@@ -427,7 +452,7 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
 
 // ---- registry -----------------------------------------------------------
 
-using TileKernel = void (*)(const CUtensorMap, const TileArgs, const TapW);
+using TileKernel = void (*)(const CUtensorMap, const TileArgs, const TapW, const CUtensorMap);
 
 struct TileInstance {
     bool sep;
