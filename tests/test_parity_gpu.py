@@ -321,3 +321,43 @@ print(json.dumps(out))
         qa = [P.quality_from_partials(a[3 * k:3 * k + 3], metric[name]) for k in range(len(a) // 3)]
         qb = [P.quality_from_partials(b[3 * k:3 * k + 3], metric[name]) for k in range(len(b) // 3)]
         np.testing.assert_allclose(qa, qb, rtol=0, atol=1e-12)
+
+
+def test_tma_store_and_register_store_epilogues_bitwise():
+    """Tile kernels send their outputs as one TMA tensor store per tile by
+    default; PARAPROX_TMA_STORE=0 keeps 128-bit register stores.  Both write
+    the same bits, including ragged edges (tiles clipped by the image) and a
+    pitched layout whose padding columns must stay untouched."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, hashlib, torch
+sys.path.insert(0, %r)
+import paper_conf_asplos_samadijlm14_b200 as pkg
+import workloads as W
+from workloads import filters as F
+P = pkg.paraprox
+h = hashlib.sha256()
+for name, w in [("gauss3", F.gaussian(3)), ("mean5", F.mean(5)), ("conv9", F.conv(9)), ("sep7", F.separable(7))]:
+    f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+    x = torch.from_numpy(W.frames(3, 131, 300, 5)).cuda()
+    r = f.ky // 2
+    for dy, dx in [(0, 0), (1, 0), (0, 1), (r, 0), (1, 1)]:
+        y = P.stencil_approx_xy(x, f, dy, dx)
+        h.update(y.cpu().numpy().tobytes())
+        xb = torch.zeros((3, 131, 308), device="cuda")
+        xb[:, :, :300] = x
+        big = torch.full((3, 131, 308), -7.0, device="cuda")
+        P.stencil_approx_xy(xb[:, :, :300], f, dy, dx, out=big[:, :, :300])
+        h.update(big.cpu().numpy().tobytes())
+print(h.hexdigest(), P.last_kernel())
+''' % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))),)
+    res = {}
+    for flag in ("1", "0"):
+        env = dict(os.environ, PARAPROX_TMA_STORE=flag)
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr
+        res[flag] = r.stdout.strip().splitlines()[-1]
+    assert res["1"] == res["0"], res
+    assert not res["1"].endswith("generic"), res
