@@ -203,11 +203,12 @@ static paraprox_status quality_partials_impl(const float* e, const float* a, con
     cudaStream_t cs = (cudaStream_t)s;
     DevBuf buf;
     buf.s = cs;
-    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * (2 * kQualityBlocks + 3), cs));
+    const size_t qsd = quality_scratch_doubles((long long)img->n * img->h * img->w);
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * (qsd + 3), cs));
     double* d = (double*)buf.p;
-    cudaError_t err = launch_quality(e, a, view_of(img), m, d + 2 * kQualityBlocks, d, cs);
+    cudaError_t err = launch_quality(e, a, view_of(img), m, d + qsd, d, cs);
     if (err != cudaSuccess) return cuda_fail(err, "quality launch");
-    PPX_CUDA(cudaMemcpyAsync(h3, d + 2 * kQualityBlocks, 3 * sizeof(double), cudaMemcpyDeviceToHost, cs));
+    PPX_CUDA(cudaMemcpyAsync(h3, d + qsd, 3 * sizeof(double), cudaMemcpyDeviceToHost, cs));
     PPX_CUDA(cudaStreamSynchronize(cs));
     return PARAPROX_OK;
 }
@@ -227,12 +228,13 @@ paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, cons
     const size_t nc = cands.size();
     DevBuf buf;
     buf.s = cs;
-    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (2 * kQualityBlocks + 3 * nc) + 256;
+    const size_t qsd = quality_scratch_doubles(count);
+    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (qsd + 3 * nc) + 256;
     PPX_CUDA(scratch_alloc(&buf.p, bytes, cs));
     float* E = (float*)buf.p;
     float* A = E + count;
     double* scratch = (double*)(((uintptr_t)(A + count) + 255) & ~(uintptr_t)255);
-    double* parts = scratch + 2 * kQualityBlocks;
+    double* parts = scratch + qsd;
     const View vin = view_of(img);
     View vq;  // compact layout of the scratch outputs
     vq.n = img->n;
@@ -279,12 +281,13 @@ static paraprox_status lattice_partials_impl(paraprox_filter f, const float* d_t
     const long long count = plane * img->n;
     DevBuf buf;
     buf.s = cs;
-    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (2 * kQualityBlocks + 3 * kLatticeCands) + 256;
+    const size_t qsd = quality_scratch_doubles(count);
+    const size_t bytes = sizeof(float) * 2 * count + sizeof(double) * (qsd + 3 * kLatticeCands) + 256;
     PPX_CUDA(scratch_alloc(&buf.p, bytes, cs));
     float* E = (float*)buf.p;
     float* A = E + count;
     double* scratch = (double*)(((uintptr_t)(A + count) + 255) & ~(uintptr_t)255);
-    double* parts = scratch + 2 * kQualityBlocks;
+    double* parts = scratch + qsd;
     const View vin = view_of(img);
     View vq;
     vq.n = img->n;
@@ -735,7 +738,7 @@ paraprox_status paraprox_quality_partials_async(const float* d_exact, const floa
     cudaStream_t cs = (cudaStream_t)s;
     DevBuf buf;
     buf.s = cs;
-    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * 2 * kQualityBlocks, cs));
+    PPX_CUDA(scratch_alloc(&buf.p, sizeof(double) * quality_scratch_doubles((long long)img->n * img->h * img->w), cs));
     cudaError_t err = launch_quality(d_exact, d_approx, view_of(img), m, d_partials3, (double*)buf.p, cs);
     if (err != cudaSuccess) return cuda_fail(err, "quality launch");
     return PARAPROX_OK;

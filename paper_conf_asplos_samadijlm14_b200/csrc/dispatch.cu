@@ -55,7 +55,8 @@ constexpr int kMaxDev = 64;
 struct Entry {
     TileInstance ti;
     bool ready[kMaxDev] = {};
-    int occ[kMaxDev] = {};
+    int occ[kMaxDev] = {};   // plain instance
+    int occq[kMaxDev] = {};  // fused-quality instance
 };
 
 std::vector<Entry>& reg() {
@@ -135,16 +136,20 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     {
         std::lock_guard<std::mutex> lk(g_mu);
         if (!e.ready[dev]) {
-            err = cudaFuncSetAttribute(e.ti.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, e.ti.smem);
-            if (err != cudaSuccess) return err;
-            int occ = 0;
-            err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, e.ti.fn, kThreads, e.ti.smem);
-            if (err != cudaSuccess) return err;
+            int occ = 0, occq = 0;
+            for (TileKernel fn : {e.ti.fn, e.ti.fnq}) {
+                err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, e.ti.smem);
+                if (err != cudaSuccess) return err;
+                err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(fn == e.ti.fn ? &occ : &occq, fn, kThreads,
+                                                                    e.ti.smem);
+                if (err != cudaSuccess) return err;
+            }
             if (!g_sms[dev]) {
                 err = cudaDeviceGetAttribute(&g_sms[dev], cudaDevAttrMultiProcessorCount, dev);
                 if (err != cudaSuccess) return err;
             }
             e.occ[dev] = occ > 0 ? occ : 1;
+            e.occq[dev] = occq > 0 ? occq : 1;
             e.ready[dev] = true;
         }
     }
@@ -189,7 +194,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
         for (int i = 0; i < p.ny; ++i)
             for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];
     }
-    long long cap = (long long)g_sms[dev] * e.occ[dev];
+    long long cap = (long long)g_sms[dev] * (qo ? e.occq[dev] : e.occ[dev]);
     if (qo && cap > kQualityBlocks) cap = kQualityBlocks;  // one partial pair per CTA
     const int grid = (int)(nt < cap ? nt : cap);
     if (qo) qo->grid = grid;
@@ -203,7 +208,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    err = cudaLaunchKernelEx(&cfg, e.ti.fn, tmap, A, W, omap);
+    err = cudaLaunchKernelEx(&cfg, qo ? e.ti.fnq : e.ti.fn, tmap, A, W, omap);
     if (err != cudaSuccess) return err;
     count_launch(qo ? "tile_quality" : e.ti.name);
     *taken = true;

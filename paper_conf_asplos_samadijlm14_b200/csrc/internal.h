@@ -130,7 +130,10 @@ cudaError_t launch_quality_final(const double* d_scratch, int g, double count, p
                                  cudaStream_t s);
 cudaError_t launch_quality(const float* e, const float* a, const View& v, paraprox_metric m,
                            double* d_part3, double* d_scratch, cudaStream_t s);
-constexpr int kQualityBlocks = 1184;  // fixed partial count -> deterministic sums
+constexpr int kQualityBlocks = 1184;  // partial-count cap of the persistent (tile, map) quality grids
+// scratch (doubles) launch_quality and launch_stencil_quality need for an
+// image of `count` pixels: one partial pair per CTA
+size_t quality_scratch_doubles(long long count);
 
 // ---- api.cpp helpers shared with runtime.cpp ----
 #define PPX_CUDA(call)                                  \

@@ -5,8 +5,8 @@
 // PAPER.md L1158-1162 Fig. 6a): the folded filter is one tap w' = sum of all
 // weights, so the stencil degenerates to the map out = w' * in -- no halo, no
 // neighbour, nothing to stage.  This kernel streams it at copy speed: each
-// thread keeps kPU = 8 independent 128-bit loads in flight (evict-first), grid =
-// resident threads, 128-bit streaming stores.  8 B of HBM per pixel.
+// CTA streams one contiguous chunk, kPU = 4 independent 128-bit loads in
+// flight per thread (evict-first), 128-bit streaming stores.  8 B of HBM per pixel.
 //
 // Rounding matches the tile kernels bit for bit: dense fmaf(w, x, 0);
 // separable fmaf(wy, fmaf(wx, x, 0), 0) (horizontal, then vertical pass).
@@ -20,6 +20,7 @@ namespace ppx {
 #define PPX_PU 4
 #endif
 constexpr int kPU = PPX_PU;
+static_assert(kPU >= 4, "quality_scratch_doubles() sizes one partial pair per 4096 floats");
 
 // streaming 128-bit load: evict-first, or with a 256-byte L2 prefetch hint
 __device__ __forceinline__ float4 ld_stream(const float4* p) {
@@ -98,38 +99,37 @@ __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict_
 }
 
 // fused quality (the tuner's centre candidates): compare w' x with the
-// reference instead of storing; 2 fp64 partials per CTA, deterministic order
+// reference instead of storing; one CTA per contiguous chunk of 256 x kPU
+// float4 (the map kernel's layout), 2 fp64 partials per CTA, deterministic
 template <bool SEP>
 __global__ void __launch_bounds__(256) k_pointwise_flat_q(const float* __restrict__ in, const float* __restrict__ ref,
                                                           long long count, float w0, float w1, int metric,
                                                           int ref_exact, double* __restrict__ part) {
     const long long n4 = count >> 2;
-    const long long stride = (long long)gridDim.x * blockDim.x;
+    const long long base = (long long)blockIdx.x * (256 * kPU) + threadIdx.x;
     const float4* i4 = reinterpret_cast<const float4*>(in);
     const float4* r4 = reinterpret_cast<const float4*>(ref);
     RAcc q;
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     auto term = [&](float v, float r) { q.add(metric, ref_exact ? r : v, ref_exact ? v : r); };
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += kPU * stride) {
-        float4 v[kPU], r[kPU];
+    float4 v[kPU], r[kPU];
 #pragma unroll
-        for (int u = 0; u < kPU; ++u)
-            if (i + u * stride < n4) {
-                v[u] = __ldcs(i4 + i + u * stride);
-                r[u] = __ldcs(r4 + i + u * stride);
-            }
+    for (int u = 0; u < kPU; ++u)
+        if (base + u * 256 < n4) {
+            v[u] = ld_stream(i4 + base + u * 256);
+            r[u] = __ldcs(r4 + base + u * 256);
+        }
 #pragma unroll
-        for (int u = 0; u < kPU; ++u)
-            if (i + u * stride < n4) {
-                const float4 a = pw4<SEP>(v[u], w0, w1);
-                term(a.x, r[u].x);
-                term(a.y, r[u].y);
-                term(a.z, r[u].z);
-                term(a.w, r[u].w);
-            }
-    }
-    if (blockIdx.x == 0)
+    for (int u = 0; u < kPU; ++u)
+        if (base + u * 256 < n4) {
+            const float4 a = pw4<SEP>(v[u], w0, w1);
+            term(a.x, r[u].x);
+            term(a.y, r[u].y);
+            term(a.z, r[u].z);
+            term(a.w, r[u].w);
+        }
+    if (blockIdx.x == gridDim.x - 1)
         for (long long x = (n4 << 2) + threadIdx.x; x < count; x += blockDim.x) term(pw<SEP>(in[x], w0, w1), ref[x]);
     double s0, s1;
     q.get(metric, s0, s1);
@@ -220,16 +220,14 @@ bool launch_pointwise_quality(const Plan& p, const float* in, const View& v, con
                       rfs == (long long)v.h * v.w)) && v.lo == 0 &&
                       (((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(ref)) & 15) == 0);
     if (!flat) return false;
-    int dev = 0, nsm = 148;
-    *err = cudaGetDevice(&dev);
-    if (*err != cudaSuccess) return true;
-    *err = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    if (*err != cudaSuccess) return true;
     const float w0 = p.separable ? p.wyf[0] : p.wf[0];
     const float w1 = p.separable ? p.wxf[0] : 1.f;
-    const long long want = (count / 4 + 255) / 256;
-    long long grid = std::min<long long>((long long)nsm * 8, kQualityBlocks);
-    grid = std::max<long long>(1, std::min(grid, want));
+    // one CTA per 256 x kPU float4 (<= quality_scratch_doubles(count) / 2 partial pairs)
+    const long long grid = std::max<long long>(1, (count / 4 + 256 * kPU - 1) / (256 * kPU));
+    if (grid >= (1LL << 31)) {
+        *err = cudaErrorInvalidValue;
+        return true;
+    }
     if (p.separable)
         k_pointwise_flat_q<true><<<(unsigned)grid, 256, 0, s>>>(in, ref, count, w0, w1, metric, ref_exact, part);
     else

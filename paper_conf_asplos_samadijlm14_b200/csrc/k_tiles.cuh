@@ -157,55 +157,42 @@ __device__ __forceinline__ void static_for(F&& f) {
     static_for_impl(f, std::make_integer_sequence<int, N>{});
 }
 
-// Out-of-line epilogue of the rarely used modes: the additive input
-// (HotSpot's power: out = acc + alpha * p + beta) and/or the fused quality
-// (compare with the reference instead of storing, accumulate into racc).
-static __device__ __noinline__ void tile_epilogue_special(const float* addp, long long apitch, long long afs, float alpha,
-                                                   float beta, const float* refp, long long rpitch, long long rfs,
-                                                   int metric, int ref_exact, float* out, long long opitch,
-                                                   long long ofs, int h, int w, int f, int yb, int x,
-                                                   const float (&r)[kRB][4], RAcc& racc) {
+// Out-of-line epilogue of the additive input (HotSpot's power: out = acc +
+// alpha * p + beta), kept out of the plain stencils' register budget.
+static __device__ __noinline__ void tile_epilogue_add(const float* addp, long long apitch, long long afs, float alpha,
+                                                      float beta, float* out, long long opitch, long long ofs, int h,
+                                                      int w, int f, int yb, int x, const float (&r)[kRB][4]) {
     for (int k = 0; k < kRB; ++k) {
         const int y = yb + k;
         if (y >= h || x >= w) continue;
         float r4[4] = {r[k][0], r[k][1], r[k][2], r[k][3]};
-        if (addp) {
-            const float* ap = addp + (long long)f * afs + x + (long long)y * apitch;
-            float a4[4] = {0.f, 0.f, 0.f, 0.f};
-            if (x + 3 < w) {
-                const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
-                a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
-            } else {
-                for (int c = 0; c < 4; ++c)
-                    if (x + c < w) a4[c] = ap[c];
-            }
-            for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(alpha, a4[c], r4[c]), beta);
-        }
-        if (refp) {
-            const float* rp = refp + (long long)f * rfs + x + (long long)y * rpitch;
-            float q4[4] = {0.f, 0.f, 0.f, 0.f};
-            if (x + 3 < w) {
-                const float4 t = __ldcs(reinterpret_cast<const float4*>(rp));
-                q4[0] = t.x, q4[1] = t.y, q4[2] = t.z, q4[3] = t.w;
-            } else {
-                for (int c = 0; c < 4; ++c)
-                    if (x + c < w) q4[c] = rp[c];
-            }
-            for (int c = 0; c < 4; ++c)
-                if (x + c < w) racc.add(metric, ref_exact ? q4[c] : r4[c], ref_exact ? r4[c] : q4[c]);
+        const float* ap = addp + (long long)f * afs + x + (long long)y * apitch;
+        float a4[4] = {0.f, 0.f, 0.f, 0.f};
+        if (x + 3 < w) {
+            const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
+            a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
         } else {
-            float* o = out + (long long)f * ofs + (long long)y * opitch + x;
-            if (x + 3 < w) {
-                __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
-            } else {
-                for (int c = 0; c < 4; ++c)
-                    if (x + c < w) __stcs(o + c, r4[c]);
-            }
+            for (int c = 0; c < 4; ++c)
+                if (x + c < w) a4[c] = ap[c];
+        }
+        for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(alpha, a4[c], r4[c]), beta);
+        float* o = out + (long long)f * ofs + (long long)y * opitch + x;
+        if (x + 3 < w) {
+            __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
+        } else {
+            for (int c = 0; c < 4; ++c)
+                if (x + c < w) __stcs(o + c, r4[c]);
         }
     }
 }
 
-template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+// Q = true: the fused-quality instance (the tuner's candidates, the runtime's
+// checks).  The thread's 8 x 4 reference values are loaded into registers at
+// the start of each tile, before the staged input is awaited, so their latency
+// hides behind the stencil's FMAs; the epilogue compares instead of storing.
+// (The first version did these loads inside an out-of-line epilogue shared
+// with the plain instance, one dependent round trip per row: 3x slower.)
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
 __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
                                                        const TileArgs A, const __grid_constant__ TapW W,
                                                        const __grid_constant__ CUtensorMap omap) {
@@ -262,7 +249,7 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             if (in_range(t)) issue(t, s);
         }
 
-    RAcc racc;  // fused-quality partials (A.refp)
+    RAcc racc;  // fused-quality partials (Q)
     int it = 0;
     for (int tile = tile_at(0); in_range(tile); tile = tile_at(++it)) {
         const int s = it % G::STAGES;
@@ -276,6 +263,27 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
         }
         int f, y0, x0;
         coords(tile, f, y0, x0);
+        const int ty0 = wi * kRB;
+        const int x = x0 + 4 * lane;
+        float4 qv[Q ? kRB : 1];  // Q: this thread's reference values, in flight during the FMAs
+        if constexpr (Q) {
+            const float* rb = A.refp + (long long)f * A.rfs + x;
+#pragma unroll
+            for (int k = 0; k < kRB; ++k) {
+                const int y = y0 + ty0 + k;
+                qv[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (y < A.h && x < A.w) {
+                    const float* rp = rb + (long long)y * A.rpitch;
+                    if (x + 3 < A.w) {
+                        qv[k] = __ldcs(reinterpret_cast<const float4*>(rp));
+                    } else {
+                        qv[k].x = rp[0];
+                        if (x + 1 < A.w) qv[k].y = rp[1];
+                        if (x + 2 < A.w) qv[k].z = rp[2];
+                    }
+                }
+            }
+        }
         float* S = reinterpret_cast<float*>(smem_raw + s * G::STAGE_STRIDE);
         mbar_wait(&bars[s], (it / G::STAGES) & 1);
 
@@ -310,7 +318,6 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             __syncthreads();
         }
 
-        const int ty0 = wi * kRB;
         // outputs as column pairs (c = 0,1 and 2,3): every FMA is a packed
         // FFMA2 (fma.rn.f32x2, sm_100) -- the same fp32 fma per lane, so the
         // per-pixel rounding and tap order are unchanged, at half the issue
@@ -385,14 +392,24 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
             }
         }
 
-        // stores: 128-bit streaming where the 4 columns are inside the image;
-        // the additive-input and fused-quality epilogues live out of line so
-        // the plain stencils keep a lean epilogue (and their register budget)
-        const int x = x0 + 4 * lane;
+        // stores: a TMA tensor store per tile or 128-bit streaming stores; the
+        // additive-input epilogue lives out of line so the plain stencils keep
+        // a lean epilogue (and their register budget)
+        if constexpr (Q) {
+#pragma unroll
+            for (int k = 0; k < kRB; ++k) {
+                const int y = y0 + ty0 + k;
+                if (y >= A.h) continue;
+                const float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
+                const float q4[4] = {qv[k].x, qv[k].y, qv[k].z, qv[k].w};
+#pragma unroll
+                for (int c = 0; c < 4; ++c)
+                    if (x + c < A.w) racc.add(A.metric, A.ref_exact ? q4[c] : r4[c], A.ref_exact ? r4[c] : q4[c]);
+            }
 #ifdef PPX_NO_SPECIAL_EPI  // A/B only: the plain store epilogue
-        if (false) {
+        } else if (false) {
 #else
-        if (A.addp || A.refp) {
+        } else if (A.addp) {
 #endif
             float r[kRB][4];
 #pragma unroll
@@ -402,8 +419,8 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
                 r[k][2] = acc[k][1].x;
                 r[k][3] = acc[k][1].y;
             }
-            tile_epilogue_special(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.refp, A.rpitch, A.rfs, A.metric,
-                                  A.ref_exact, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0, x, r, racc);
+            tile_epilogue_add(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0,
+                              x, r);
         } else if (A.tma_store) {
             // the tile's outputs replace its consumed input stage ([kTH][kTW])
             // and leave as one TMA store (out-of-image elements are clipped)
@@ -439,7 +456,7 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
         __syncthreads();  // stage s fully consumed before it is refilled
     }
     if (A.tma_store && tid == 0) bulk_wait_all();
-    if (A.refp) {  // deterministic: fixed tile order per CTA, fixed reduction tree
+    if constexpr (Q) {  // deterministic: fixed tile order per CTA, fixed reduction tree
         double s0, s1;
         racc.get(A.metric, s0, s1);
         block_sum2(s0, s1);
@@ -458,7 +475,8 @@ struct TileInstance {
     bool sep;
     uint32_t masky, maskx;
     int hy, hx;
-    TileKernel fn;
+    TileKernel fn;   // plain / additive-input stencil
+    TileKernel fnq;  // fused-quality instance
     int smem;
     const char* name;
 };
@@ -473,7 +491,8 @@ TileInstance make_instance(const char* name) {
     ti.maskx = MASKX;
     ti.hy = HY;
     ti.hx = HX;
-    ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP>;
+    ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP, false>;
+    ti.fnq = k_tiles<HY, HX, MASKY, MASKX, SEP, true>;
     ti.smem = Geom<HY, HX>::SMEM;
     ti.name = name;
     return ti;

@@ -259,7 +259,7 @@ paraprox_status paraprox_runtime_run(paraprox_runtime rt, const float* d_in, flo
         if (!rt->h_part) PPX_CUDA(cudaMallocHost(&rt->h_part, 3 * sizeof(double)));
         if (!rt->ev) PPX_CUDA(cudaEventCreateWithFlags(&rt->ev, cudaEventDisableTiming));
         void* scratch = nullptr;
-        PPX_CUDA(scratch_alloc(&scratch, sizeof(double) * 2 * kQualityBlocks, cs));
+        PPX_CUDA(scratch_alloc(&scratch, sizeof(double) * quality_scratch_doubles((long long)img->n * img->h * img->w), cs));
         bool fused = false;
         cudaError_t e = launch_stencil_quality(get_plan(rt->f, 0, 0), d_in, view_of(img), d_out, img->pitch, ofs0,
                                                rt->m, false, rt->d_part, (double*)scratch, cs, &fused);
@@ -301,7 +301,7 @@ paraprox_status paraprox_runtime_run(paraprox_runtime rt, const float* d_in, flo
     vq.lo = 0;
     vq.hi = img->h - 1;
     void* scratch = nullptr;
-    PPX_CUDA(scratch_alloc(&scratch, sizeof(double) * 2 * kQualityBlocks, cs));
+    PPX_CUDA(scratch_alloc(&scratch, sizeof(double) * quality_scratch_doubles((long long)img->n * img->h * img->w), cs));
     e = launch_quality(rt->d_exact, d_out, vq, rt->m, rt->d_part, (double*)scratch, cs);
     cudaFreeAsync(scratch, cs);
     if (e != cudaSuccess) return cuda_fail(e, "check quality launch");
