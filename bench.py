@@ -532,6 +532,8 @@ def main():
         def quality_step(k):
             P.quality_partials_async(outputs[k % nbuf], inputs[k % nbuf], wl["metric"], qpart, stream=stream)
 
+        # eager: its per-call scratch (cudaMallocAsync) would become graph
+        # memory nodes, measured slower on replay (c2: 36.6 vs 26.5 us)
         qual_ms, qual_kern_ms, _ = timed(quality_step, args.steps, args.warmup)
 
         # NEXT-1: the global-lattice reading (only every (2d+1)-th row is read
@@ -698,7 +700,7 @@ def main():
             "quality_kernel": {"metric": wl["metric"], "ms": qual_kern_ms, "kernel": "quality_flat",
                                "achieved_gbs": alg_bytes / (qual_kern_ms * 1e-3) / 1e9,
                                "frac": alg_bytes / (qual_kern_ms * 1e-3) / 1e9 / peak,
-                               "note": "a4 alone: reads E and A (8 B/px), fp64 partials, 2 launches"},
+                               "note": "a4 alone: reads E and A (8 B/px), fp64 partials; partial + final kernels (PDL), eager"},
             "lattice": lat,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "frac_of_nominal_8tbs": achieved / 8000.0, "traffic": load_traffic(args.workload, approx_kernel),

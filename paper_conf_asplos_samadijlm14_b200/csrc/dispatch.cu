@@ -193,6 +193,8 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     } else {
         for (int i = 0; i < p.ny; ++i)
             for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];
+        for (int a = -3; a <= 4; ++a)  // row-pair weights (k_tiles.cuh, use_row_pairs)
+            for (int b = 0; b < 9; ++b) W.wp[a + 4][b] = make_float2(W.w[a + 4][b], W.w[a + 3][b]);
     }
     long long cap = (long long)g_sms[dev] * (qo ? e.occq[dev] : e.occ[dev]);
     if (qo && cap > kQualityBlocks) cap = kQualityBlocks;  // one partial pair per CTA

@@ -10,6 +10,31 @@
 
 namespace ppx {
 
+// Programmatic dependent launch: every quality kernel is launched with
+// programmatic stream serialisation, so its CTAs may be scheduled while the
+// previous kernel on the stream (a stencil, or the previous reduction level)
+// drains.  griddepcontrol.wait blocks until that kernel has completed and its
+// writes are visible; launch_dependents then lets the next level be scheduled
+// early in turn.  Both are no-ops for a plain launch.
+__device__ __forceinline__ void pdl_wait_and_release() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*k)(KArgs...), int grid, int block, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 // Contiguous images (pitch == w, frames back to back) are one flat array:
 // one CTA per contiguous chunk of 256 x kQU float4 of E and of A (all loads of
 // a thread issued before any arithmetic), one partial pair per CTA.  The
@@ -27,6 +52,7 @@ static_assert(kQU >= 4, "quality_scratch_doubles() sizes one partial pair per 40
 template <int M>
 __global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ E, const float* __restrict__ A,
                                                       long long count, double* __restrict__ part) {
+    pdl_wait_and_release();
     QAcc<M> q;
     const long long n4 = count >> 2;
     const long long base = (long long)blockIdx.x * (256 * kQU) + threadIdx.x;
@@ -71,6 +97,7 @@ template <int M>
 __global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_partials(const float* __restrict__ E,
                                                           const float* __restrict__ A, View v,
                                                           double* __restrict__ part) {
+    pdl_wait_and_release();
     QAcc<M> q;
     const long long rows = (long long)v.n * v.h;
     const bool vec = ((v.pitch & 3) == 0) && ((v.fstride & 3) == 0) &&
@@ -121,6 +148,7 @@ __global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_part
 template <int M>
 __global__ void __launch_bounds__(1024) k_quality_final(const double* __restrict__ part, int g,
                                                         double count, double* __restrict__ out3) {
+    pdl_wait_and_release();
     double s0 = 0.0, s1 = 0.0;
     for (int k = threadIdx.x; k < g; k += blockDim.x) {
         s0 += part[2 * k];
@@ -156,15 +184,17 @@ cudaError_t launch_quality(const float* e, const float* a, const View& v, parapr
     } else {
         g = (int)(rows < kQualityBlocks ? rows : kQualityBlocks);
     }
+    cudaError_t err;
 #define PPX_QUALITY_CASE(M)                                                                    \
-    if (flat) k_quality_flat<M><<<g, 256, 0, s>>>(e, a, cnt, d_scratch);                       \
-    else k_quality_partials<M><<<g, 256, 0, s>>>(e, a, v, d_scratch);
+    if (flat) err = launch_pdl(k_quality_flat<M>, g, 256, s, e, a, cnt, d_scratch);            \
+    else err = launch_pdl(k_quality_partials<M>, g, 256, s, e, a, v, d_scratch);
     switch (m) {
     case PARAPROX_MRE: PPX_QUALITY_CASE(PARAPROX_MRE) break;
     case PARAPROX_L2: PPX_QUALITY_CASE(PARAPROX_L2) break;
     default: PPX_QUALITY_CASE(PARAPROX_PSNR) break;
     }
 #undef PPX_QUALITY_CASE
+    if (err != cudaSuccess) return err;
     count_launch(flat ? "quality_flat" : "quality_partials");
     return launch_quality_final(d_scratch, g, count, m, d_part3, s);
 }
@@ -175,6 +205,7 @@ cudaError_t launch_quality(const float* e, const float* a, const View& v, parapr
 constexpr int kFold = 2048;
 __global__ void __launch_bounds__(256) k_quality_fold(const double* __restrict__ part, int g,
                                                       double* __restrict__ out) {
+    pdl_wait_and_release();
     double s0 = 0.0, s1 = 0.0;
     const int k0 = blockIdx.x * kFold;
     const int k1 = min(g, k0 + kFold);
@@ -196,16 +227,19 @@ cudaError_t launch_quality_final(const double* d_scratch, int g, double count, p
     if (g > 2 * kFold) {
         double* lvl2 = const_cast<double*>(d_scratch) + 2 * (size_t)g;
         const int g2 = (g + kFold - 1) / kFold;
-        k_quality_fold<<<g2, 256, 0, s>>>(d_scratch, g, lvl2);
+        cudaError_t err = launch_pdl(k_quality_fold, g2, 256, s, d_scratch, g, lvl2);
+        if (err != cudaSuccess) return err;
         count_launch("quality_fold");
         d_scratch = lvl2;
         g = g2;
     }
+    cudaError_t err;
     switch (m) {
-    case PARAPROX_MRE: k_quality_final<PARAPROX_MRE><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
-    case PARAPROX_L2: k_quality_final<PARAPROX_L2><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
-    default: k_quality_final<PARAPROX_PSNR><<<1, 1024, 0, s>>>(d_scratch, g, count, d_part3); break;
+    case PARAPROX_MRE: err = launch_pdl(k_quality_final<PARAPROX_MRE>, 1, 1024, s, d_scratch, g, count, d_part3); break;
+    case PARAPROX_L2: err = launch_pdl(k_quality_final<PARAPROX_L2>, 1, 1024, s, d_scratch, g, count, d_part3); break;
+    default: err = launch_pdl(k_quality_final<PARAPROX_PSNR>, 1, 1024, s, d_scratch, g, count, d_part3); break;
     }
+    if (err != cudaSuccess) return err;
     count_launch("quality_final");
     return cudaGetLastError();
 }

@@ -54,6 +54,10 @@ constexpr int kTH = kRB * kWarps;        // 64 tile rows
 constexpr int kThreads = 32 * kWarps;
 
 struct TapW {
+    // row-pair weights for the row-pair form (below): wp[a + 4][b + 4] =
+    // (w[a][b], w[a - 1][b]), the taps of offset (., b) that input row y + a
+    // feeds into output rows (y, y + 1); filled for a in [-3, 4]
+    float2 wp[9][9];
     float w[9][9];   // dense folded weights at [a + 4][b + 4]   (r <= 4)
     float wy[17];    // separable folded weights at [a + 8]     (r <= 8)
     float wx[17];
@@ -192,6 +196,30 @@ static __device__ __noinline__ void tile_epilogue_add(const float* addp, long lo
 // hides behind the stencil's FMAs; the epilogue compares instead of storing.
 // (The first version did these loads inside an out-of-line epilogue shared
 // with the plain instance, one dependent round trip per row: 3x slower.)
+// Row-pair form of the dense stencil.  The column-pair form packs a thread's
+// outputs (x, x+1) and (x+2, x+3) into FFMA2 lanes, so every odd column offset
+// b needs the pair (v[x+b], v[x+b+1]) straddling two 64-bit registers: ptxas
+// builds it with MOVs (882 per tile at the exact 9x9, as many issue slots as
+// 2/3 of the FFMA2s).  The row-pair form packs output rows (y, y+1) of one
+// column instead: the staged input value is the broadcast scalar operand of
+// FFMA2 and the weight pair (w[a][b], w[a-1][b]) comes from the parameter bank
+// as a uniform register pair, so no operand is ever rebuilt.  The first and
+// last input rows of a pair feed only one of its rows: a scalar FFMA on that
+// half.  Per-pixel tap order (input row, then column offset) and the fp32 fma
+// per tap are unchanged, so outputs are bit-identical to the column-pair form.
+// Used when the accessed rows are contiguous (pairs of rows both accessed)
+// and some column offset is odd (else the column-pair form has no MOVs).
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX>
+__host__ __device__ constexpr bool use_row_pairs() {
+    bool full = HY >= 1, odd = false;
+    for (int a = -HY; a <= HY; ++a) full = full && ((MASKY >> (a + 8)) & 1u);
+    for (int b = -HX; b <= HX; ++b) odd = odd || (((MASKX >> (b + 8)) & 1u) && (b & 1));
+#ifdef PPX_NO_ROW_PAIRS  // A/B only
+    full = false;
+#endif
+    return full && odd;
+}
+
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
 __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
                                                        const TileArgs A, const __grid_constant__ TapW W,
@@ -326,7 +354,53 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
 #pragma unroll
         for (int k = 0; k < kRB; ++k) acc[k][0] = acc[k][1] = make_float2(0.f, 0.f);
 
-        if constexpr (!SEP) {
+        if constexpr (!SEP && use_row_pairs<HY, HX, MASKY, MASKX>()) {
+            float2 rp[kRB / 2][4];  // rp[p][c] = outputs (rows 2p, 2p+1) of column c
+#pragma unroll
+            for (int p = 0; p < kRB / 2; ++p)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) rp[p][c] = make_float2(0.f, 0.f);
+            static_for<kRB + 2 * HY>([&](auto RR) {
+                constexpr int rr = decltype(RR)::value;
+                const int sr = min(max(ty0 + rr, rlo), rhi);
+                float v[NV];
+                const float4* p4 = reinterpret_cast<const float4*>(S + sr * SW) + lane;
+#pragma unroll
+                for (int q = 0; q < NV / 4; ++q) {
+                    const float4 t = p4[q];
+                    v[4 * q] = t.x, v[4 * q + 1] = t.y, v[4 * q + 2] = t.z, v[4 * q + 3] = t.w;
+                }
+                static_for<kRB / 2>([&](auto KP) {
+                    constexpr int p = decltype(KP)::value;
+                    constexpr int a0 = rr - HY - 2 * p, a1 = a0 - 1;  // offsets for rows 2p, 2p+1
+                    constexpr bool u0 = a0 >= -HY && a0 <= HY, u1 = a1 >= -HY && a1 <= HY;
+                    if constexpr (u0 || u1) {
+                        static_for<2 * HX + 1>([&](auto B) {
+                            constexpr int b = decltype(B)::value - HX;
+                            if constexpr (has(MASKX, b)) {
+#pragma unroll
+                                for (int c = 0; c < 4; ++c) {
+                                    const float xv = v[HXP + b + c];
+                                    if constexpr (u0 && u1)
+                                        rp[p][c] = __ffma2_rn(W.wp[a0 + 4][b + 4], make_float2(xv, xv), rp[p][c]);
+                                    else if constexpr (u0)
+                                        rp[p][c].x = __fmaf_rn(W.w[a0 + 4][b + 4], xv, rp[p][c].x);
+                                    else
+                                        rp[p][c].y = __fmaf_rn(W.w[a1 + 4][b + 4], xv, rp[p][c].y);
+                                }
+                            }
+                        });
+                    }
+                });
+            });
+#pragma unroll
+            for (int p = 0; p < kRB / 2; ++p) {
+                acc[2 * p][0] = make_float2(rp[p][0].x, rp[p][1].x);
+                acc[2 * p][1] = make_float2(rp[p][2].x, rp[p][3].x);
+                acc[2 * p + 1][0] = make_float2(rp[p][0].y, rp[p][1].y);
+                acc[2 * p + 1][1] = make_float2(rp[p][2].y, rp[p][3].y);
+            }
+        } else if constexpr (!SEP) {
             // fully unrolled at compile time (static_for): the weights are
             // kernel-parameter constants at fixed offsets, no indexed loads
             static_for<kRB + 2 * HY>([&](auto RR) {
