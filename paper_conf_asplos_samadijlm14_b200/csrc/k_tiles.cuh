@@ -138,13 +138,29 @@ __device__ __forceinline__ void load_pairs(const float* row, int lane, float2 (&
 }
 
 // acc[0] += w * (v[I0], v[I0+1]); acc[1] += w * (v[I0+2], v[I0+3])
-template <int NV, int I0>
+// Even I0: two FFMA2 on register pairs straight from LDS.128.  Odd I0: the
+// pairs (v[I0], v[I0+1]) straddle two 64-bit registers; ptxas builds them
+// with MOVs, which take FMA-pipe cycles of their own (ncu), so four scalar
+// FFMAs -- the same issue slots, fewer pipe cycles, same fp32 fma per lane --
+// are used instead (PPX_ODD_PAIRS=1 keeps the pair form, A/B; kbench at c4
+// and c3: lattice +4-12 %, separable exact +21 %, dense column-pair instances
+// within +-5 % except dense_l3_f4, 14 % slower, which keeps the pair form).
+#ifndef PPX_ODD_PAIRS
+#define PPX_ODD_PAIRS 0
+#endif
+template <int NV, int I0, bool ODD_PAIRS = PPX_ODD_PAIRS>
 __device__ __forceinline__ void fma_pairs(float2 (&acc)[2], float w, const float2 (&ve)[NV / 2],
                                           const float2 (&vo)[NV / 2 - 1]) {
     const float2 w2 = make_float2(w, w);
     if constexpr ((I0 & 1) == 0) {
         acc[0] = __ffma2_rn(w2, ve[I0 >> 1], acc[0]);
         acc[1] = __ffma2_rn(w2, ve[(I0 >> 1) + 1], acc[1]);
+    } else if constexpr (!ODD_PAIRS) {
+        // v[I0] = ve[I0/2].y, v[I0+1] = ve[I0/2+1].x, ...
+        acc[0].x = __fmaf_rn(w, ve[I0 >> 1].y, acc[0].x);
+        acc[0].y = __fmaf_rn(w, ve[(I0 >> 1) + 1].x, acc[0].y);
+        acc[1].x = __fmaf_rn(w, ve[(I0 >> 1) + 1].y, acc[1].x);
+        acc[1].y = __fmaf_rn(w, ve[(I0 >> 1) + 2].x, acc[1].y);
     } else {
         acc[0] = __ffma2_rn(w2, vo[I0 >> 1], acc[0]);
         acc[1] = __ffma2_rn(w2, vo[(I0 >> 1) + 1], acc[1]);
@@ -218,6 +234,13 @@ __host__ __device__ constexpr bool use_row_pairs() {
     full = false;
 #endif
     return full && odd;
+}
+
+// the one instance the odd-offset A/B measured faster with the pair form
+// (fma_pairs): dense rows {-3, 0, 3} x columns {-4..4}
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX>
+__host__ __device__ constexpr bool odd_pairs_faster() {
+    return HY == 3 && HX == 4 && MASKY == ((1u << 5) | (1u << 8) | (1u << 11)) && MASKX == (0x1FFu << 4);
 }
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
@@ -415,7 +438,9 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
                         if constexpr (a >= -HY && a <= HY && has(MASKY, a)) {
                             static_for<2 * HX + 1>([&](auto B) {
                                 constexpr int b = decltype(B)::value - HX;
-                                if constexpr (has(MASKX, b)) fma_pairs<NV, HXP + b>(acc[k], W.w[a + 4][b + 4], ve, vo);
+                                if constexpr (has(MASKX, b))
+                                    fma_pairs<NV, HXP + b, PPX_ODD_PAIRS || odd_pairs_faster<HY, HX, MASKY, MASKX>()>(
+                                        acc[k], W.w[a + 4][b + 4], ve, vo);
                             });
                         }
                     });
