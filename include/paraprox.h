@@ -267,9 +267,11 @@ PARAPROX_API paraprox_status paraprox_quality_from_partials(const double* h_part
 
 /* The runtime tuner (L572-592; L1220-1226; training on the first frames,
  * L1620-1628): the exact kernel runs once on the training frames d_train,
- * every candidate (scheme, reach) in cost order runs and is scored; the
- * first candidate with quality >= toq is returned, else (EXACT, 0, 1.0 or
- * +inf dB).  toq in (0, 1] for MRE / L2; any value (dB) for PSNR. */
+ * then the candidates (scheme, reach) run in cost order, each scored against
+ * it; the first candidate with quality >= toq is returned (the scan stops
+ * there: one stream sync per candidate scored), else (EXACT, 0, 1.0 or
+ * +inf dB).  toq in (0, 1] for MRE / L2; any value (dB) for PSNR.  The
+ * decision equals paraprox_tune_decide on paraprox_tune_partials' full scan. */
 PARAPROX_API paraprox_status paraprox_tune(paraprox_filter f, const float* d_train, const paraprox_image* img,
                               double toq, paraprox_metric m, paraprox_scheme* out_scheme,
                               int* out_reach, double* out_quality, paraprox_stream s);

@@ -216,7 +216,7 @@ static paraprox_status quality_partials_impl(const float* e, const float* a, con
 // all candidates' partials into h_partials[3 * n]
 paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
                                           paraprox_metric m, const std::vector<Candidate>& cands,
-                                          double* h_partials, paraprox_stream s) {
+                                          double* h_partials, paraprox_stream s, double stop_toq) {
     if (!f || !d_train || (!h_partials && !cands.empty())) return fail(PARAPROX_ERR_INVALID_ARG, "NULL pointer");
     if (!metric_ok(m)) return fail(PARAPROX_ERR_INVALID_ARG, "unknown metric");
     paraprox_status st = check_image(img, true);
@@ -255,12 +255,25 @@ paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, cons
                                        parts + 3 * k, scratch, cs, &fused);
             if (e != cudaSuccess) return cuda_fail(e, "fused candidate launch");
         }
-        if (fused) continue;
-        e = launch_stencil(cand_plan(f, cands[k]), d_train, vin, A, img->w, plane, cs);
-        if (e != cudaSuccess) return cuda_fail(e, "candidate launch");
-        e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);
-        if (e != cudaSuccess) return cuda_fail(e, "quality launch");
+        if (!fused) {
+            e = launch_stencil(cand_plan(f, cands[k]), d_train, vin, A, img->w, plane, cs);
+            if (e != cudaSuccess) return cuda_fail(e, "candidate launch");
+            e = launch_quality(E, A, vq, m, parts + 3 * k, scratch, cs);
+            if (e != cudaSuccess) return cuda_fail(e, "quality launch");
+        }
+        if (!std::isnan(stop_toq)) {
+            // early exit (paraprox_tune): the decision is the first candidate
+            // in cost order with Q >= TOQ, so nothing after it is needed; the
+            // partials of candidates 0..k are the same bits as in a full scan
+            PPX_CUDA(cudaMemcpyAsync(h_partials + 3 * k, parts + 3 * k, sizeof(double) * 3, cudaMemcpyDeviceToHost, cs));
+            PPX_CUDA(cudaStreamSynchronize(cs));
+            if (quality_of(h_partials + 3 * k, m) >= stop_toq) {
+                for (size_t j = k + 1; j < nc; ++j) h_partials[3 * j] = h_partials[3 * j + 1] = h_partials[3 * j + 2] = NAN;
+                return PARAPROX_OK;
+            }
+        }
     }
+    if (!std::isnan(stop_toq)) return PARAPROX_OK;  // every candidate copied above
     PPX_CUDA(cudaMemcpyAsync(h_partials, parts, sizeof(double) * 3 * nc, cudaMemcpyDeviceToHost, cs));
     PPX_CUDA(cudaStreamSynchronize(cs));
     return PARAPROX_OK;
@@ -807,7 +820,7 @@ paraprox_status paraprox_tune_ex(paraprox_filter f, int flags, const float* d_tr
     if (st != PARAPROX_OK) return st;
     std::vector<Candidate> c = candidates_ex(f, flags);
     std::vector<double> parts(3 * c.size() + 3);
-    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s);
+    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s, toq);
     if (st != PARAPROX_OK) return st;
     return decide(c, parts.data(), m, toq, out_scheme, out_reach, out_quality);
 }
@@ -836,7 +849,7 @@ paraprox_status paraprox_tune(paraprox_filter f, const float* d_train, const par
     if (st != PARAPROX_OK) return st;
     std::vector<Candidate> c = candidates(f);
     std::vector<double> parts(3 * c.size() + 3);
-    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s);
+    st = tune_partials_impl(f, d_train, img, m, c, parts.data(), s, toq);
     if (st != PARAPROX_OK) return st;
     return decide(c, parts.data(), m, toq, out_scheme, out_reach, out_quality);
 }
@@ -863,9 +876,12 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     float* din = (float*)buf.p;
     float* dout = din + plane * n;
     // chunks: frames when batched, else row bands (halo rows come along);
-    // ~8 MiB per chunk (fill and drain of the copy pipeline are one chunk each), at most 16
+    // ~8 MiB per chunk, at most 64: fill and drain of the copy pipeline are
+    // one chunk each (16 chunks left c3's 8.5 GB at 0.95 of the PCIe bound,
+    // 64 reach it), and each chunk costs ~30 us of host calls (2 MiB chunks
+    // made c2's 64 MiB 30 % slower than 8 MiB ones)
     const long long total_bytes = (long long)sizeof(float) * plane * n;
-    const int want = (int)std::min<long long>(16, std::max<long long>(1, total_bytes >> 23));
+    const int want = (int)std::min<long long>(64, std::max<long long>(1, total_bytes >> 23));
     const int chunks = n > 1 ? std::min(n, want) : std::max(1, std::min(want, h / 64));
     // copy streams and events are created once per thread and device, reused
     struct Pipe {

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <atomic>
+#include <cmath>
 #include <cstdint>
 #include <map>
 #include <mutex>
@@ -155,7 +156,8 @@ paraprox_status check_toq(double toq, paraprox_metric m);
 cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s);
 paraprox_status tune_partials_impl(paraprox_filter f, const float* d_train, const paraprox_image* img,
                                    paraprox_metric m, const std::vector<Candidate>& cands, double* h_partials,
-                                   paraprox_stream s);
+                                   paraprox_stream s,
+                                   double stop_toq = NAN);
 
 // TMA-store epilogues of the tile and lattice kernels (default on);
 // PARAPROX_TMA_STORE=0 keeps 128-bit register stores (A/B, and
