@@ -25,6 +25,7 @@
 //  * Outputs leave as 128-bit streaming stores (st.global.cs).
 #pragma once
 
+#include <climits>
 #include <type_traits>
 #include <utility>
 
@@ -90,6 +91,10 @@ struct TileArgs {
     // plain stencils: outputs leave as one TMA store per tile (omap) instead
     // of 128-bit register stores (PARAPROX_TMA_STORE=0 selects the latter)
     int tma_store;
+    // tile schedule: CTA b takes tiles base + k * stride, k < chunk, with
+    // base = (b / stride) * stride * chunk + b % stride (stride = the resident
+    // CTAs); chunk = INT_MAX is the fully persistent grid (b + k * gridDim)
+    int stride, chunk;
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -285,14 +290,26 @@ __global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const _
     // the CTA's k-th tile: strided (b + k G: concurrently running CTAs take
     // neighbouring tiles) or, with PPX_TILE_RUNS, a contiguous run of tiles
     // along the rows (a tile's left halo was fetched by the same CTA just before)
+    //
+    // Bounded persistence (A.chunk < INT_MAX): a fully persistent grid lets
+    // its CTAs drift apart over hundreds of tiles, so the tiles in flight no
+    // longer form one compact window and the neighbours' halo rows and columns
+    // miss in L2 (c3, 882 tiles per CTA: DRAM reads 1.32x the input).  With
+    // chunks, each CTA takes `chunk` tiles of the stride pattern and retires;
+    // the block scheduler starts the next wave's CTAs in order as slots free
+    // up, which keeps the window compact.
 #if PPX_TILE_RUNS
     const int per = (A.ntiles + gridDim.x - 1) / gridDim.x;
     const int t_begin = blockIdx.x * per, t_end = min(A.ntiles, t_begin + per);
     auto tile_at = [&](int k) { return t_begin + k; };
     auto in_range = [&](int t) { return t < t_end; };
 #else
-    auto tile_at = [&](int k) { return (int)blockIdx.x + k * (int)gridDim.x; };
-    auto in_range = [&](int t) { return t < A.ntiles; };
+    const int wave = (int)blockIdx.x / A.stride;
+    const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
+    const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
+                                               : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
+    auto tile_at = [&](int k) { return (int)min(t_base + (long long)k * A.stride, (long long)INT_MAX); };
+    auto in_range = [&](int t) { return t < t_end; };
 #endif
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s) {
