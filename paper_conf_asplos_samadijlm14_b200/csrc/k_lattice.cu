@@ -24,6 +24,7 @@
 // Column / centre lattices (no DRAM saving: a 32-byte sector holds 8 floats)
 // and other shapes take k_lattice_generic: one thread per output, K_y x K_x
 // gathered loads of X(g(clamp(y+i)), g(clamp(x+j))).
+#include <climits>
 #include <cstdlib>
 #include <mutex>
 
@@ -71,6 +72,7 @@ struct LatArgs {
     int tiles_x, tiles_y, ntiles;
     float* out;
     long long opitch, ofs;
+    int stride, chunk;  // tile schedule, as TileArgs (bounded persistence)
 };
 
 struct LatW {
@@ -114,18 +116,24 @@ __global__ void __launch_bounds__(kThreads, PPX_LAT_MIN_BLOCKS) k_lattice(const 
     __syncthreads();
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    // CTA b takes tiles t_base + k * stride, k < chunk (k_tiles.cuh)
+    const int wave = (int)blockIdx.x / A.stride;
+    const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
+    const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
+                                               : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s) {
-            const int t = blockIdx.x + s * gridDim.x;
-            if (t < A.ntiles) issue(t, s);
+            const long long t = t_base + (long long)s * A.stride;
+            if (t < t_end) issue((int)t, s);
         }
 
     int it = 0;
-    for (int tile = blockIdx.x; tile < A.ntiles; tile += gridDim.x, ++it) {
+    for (long long tl = t_base; tl < t_end; tl += A.stride, ++it) {
+        const int tile = (int)tl;
         const int s = it % G::STAGES;
         if (tid == 0) {
-            const int ahead = tile + (G::STAGES - 1) * gridDim.x;
-            if (ahead < A.ntiles) issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+            const long long ahead = tl + (long long)(G::STAGES - 1) * A.stride;
+            if (ahead < t_end) issue((int)ahead, (it + G::STAGES - 1) % G::STAGES);
         }
         int f, y0, x0;
         coords(tile, f, y0, x0);
@@ -305,6 +313,20 @@ static const LatInstance* find_lat(int s, int r, bool sep) {
     return nullptr;
 }
 
+// tiles per CTA (bounded persistence, k_tiles.cuh); PARAPROX_LATTICE_CHUNK=0
+// keeps the fully persistent grid
+#ifndef PPX_LAT_CHUNK_DEFAULT
+#define PPX_LAT_CHUNK_DEFAULT 8
+#endif
+static int lattice_chunk() {
+    static const int v = [] {
+        const char* e = std::getenv("PARAPROX_LATTICE_CHUNK");
+        const int c = e ? std::atoi(e) : PPX_LAT_CHUNK_DEFAULT;
+        return c > 0 ? c : INT_MAX;
+    }();
+    return v;
+}
+
 static bool lattice_force_generic() {
     static int v = -1;
     if (v < 0) {
@@ -406,8 +428,16 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
     if (lf.separable)
         for (int j = 0; j < lf.kx; ++j) W.wx[j - r + 4] = lf.wx[j];
     const long long cap = (long long)nsm * occ;
+    long long grid = nt < cap ? nt : cap;
+    A.stride = (int)grid;
+    A.chunk = lattice_chunk();
+    if (A.chunk != INT_MAX) {
+        const long long waves = (nt + grid * A.chunk - 1) / (grid * A.chunk);
+        if (waves * grid >= (1LL << 31)) return launch_lattice_generic(lf, in, v, out, opitch, ofs, dy, dx, s);
+        grid *= waves;
+    }
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)(nt < cap ? nt : cap));
+    cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(kThreads);
     cfg.dynamicSmemBytes = e->smem;
     cfg.stream = s;
