@@ -140,12 +140,28 @@ def oracle_run(x, kind, w, scheme, reach):
     return oracle.stencil_approx(x, w, scheme, reach)
 
 
+def oracle_host_threads():
+    """The host cores this process may use, given to the oracle's OpenMP
+    runtime.  Under torchrun every rank gets OMP_NUM_THREADS=1, but the
+    oracle legs run on rank 0 alone while the other ranks idle."""
+    import ctypes
+    import oracle
+    n = len(os.sched_getaffinity(0))
+    os.environ["OMP_NUM_THREADS"] = str(n)  # before liboracle (and its libgomp) loads
+    oracle.lib()
+    try:
+        ctypes.CDLL("libgomp.so.1").omp_set_num_threads(n)
+    except OSError:
+        pass
+    return n
+
+
 def cpu_baseline(wl, kind, w, scheme, reach, budget_s=10.0, max_reps=400):
     """The oracle as it stands, on the host cores, over a bounded sample of the
     workload: whole frames (or a row band of the c4 image) until ~budget_s."""
     import oracle
     import workloads as W
-    cores = int(os.environ.get("OMP_NUM_THREADS", len(os.sched_getaffinity(0))))
+    cores = oracle_host_threads()
     h, wd = wl["h"], wl["w"]
     rows = h if h * wd <= 4096 * 4096 else 1024
     x = W.image(rows, wd, 1000) if rows == h else W.periodic(rows, wd, tile=4096, seed=0)
@@ -195,7 +211,7 @@ def run_reference(args):
     import oracle
     wl = WORKLOADS[args.workload]
     kind, w = make_filter_arrays(wl["filter"])
-    cores = int(os.environ.get("OMP_NUM_THREADS", len(os.sched_getaffinity(0))))
+    cores = oracle_host_threads()
     # bounded sample per step: a 512-row band of the frame, at the scheme the
     # oracle tuner picks at the TOQ on a small training set (2 frames, 512 rows)
     band = min(wl["h"], 512)

@@ -875,14 +875,36 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
     PPX_CUDA(scratch_alloc(&buf.p, sizeof(float) * 2 * plane * n, cs));
     float* din = (float*)buf.p;
     float* dout = din + plane * n;
-    // chunks: frames when batched, else row bands (halo rows come along);
-    // ~8 MiB per chunk, at most 64: fill and drain of the copy pipeline are
-    // one chunk each (16 chunks left c3's 8.5 GB at 0.95 of the PCIe bound,
-    // 64 reach it), and each chunk costs ~30 us of host calls (2 MiB chunks
-    // made c2's 64 MiB 30 % slower than 8 MiB ones)
-    const long long total_bytes = (long long)sizeof(float) * plane * n;
-    const int want = (int)std::min<long long>(64, std::max<long long>(1, total_bytes >> 23));
-    const int chunks = n > 1 ? std::min(n, want) : std::max(1, std::min(want, h / 64));
+    // chunks: frames when batched, else row bands of >= 64 rows (halo rows
+    // come along).  ~8 MiB per chunk, at most 64: each chunk costs ~30 us of
+    // host calls (2 MiB chunks made c2's 64 MiB 30 % slower than 8 MiB ones).
+    // The pipeline's fill (first upload) and drain (last download) are not
+    // overlapped, so the chunks ramp up and down (1/8, 1/4, 1/2 of the target
+    // at both ends) when there is room: uniform 8 MiB chunks left c2's 64 MiB
+    // at ~0.8 of the PCIe duplex bound.
+    const long long units = n > 1 ? n : h;
+    const long long unit_bytes = (long long)sizeof(float) * (n > 1 ? plane : w);
+    const long long min_units = n > 1 ? 1 : std::min<long long>(h, 64);
+    long long target = std::max(min_units, (8LL << 20) / std::max(1LL, unit_bytes));
+    target = std::max(target, (units + 63) / 64);
+    std::vector<long long> bounds(1, 0);
+    {
+        const long long r[3] = {std::max(min_units, target / 8), std::max(min_units, target / 4),
+                                std::max(min_units, target / 2)};
+        const long long ramp = r[0] + r[1] + r[2];
+        if (2 * ramp + target <= units && target > r[2]) {
+            for (long long q : r) bounds.push_back(bounds.back() + q);
+            const long long mid = units - 2 * ramp;
+            const long long nm = std::max(1LL, (mid + target - 1) / target);
+            const long long b0 = bounds.back();
+            for (long long c = 1; c <= nm; ++c) bounds.push_back(b0 + mid * c / nm);
+            for (int k = 2; k >= 0; --k) bounds.push_back(bounds.back() + r[k]);
+        } else {
+            const long long nc = std::max(1LL, std::min(units / min_units, (units + target - 1) / target));
+            for (long long c = 1; c <= nc; ++c) bounds.push_back(units * c / nc);
+        }
+    }
+    const int chunks = (int)bounds.size() - 1;
     // copy streams and events are created once per thread and device, reused
     struct Pipe {
         int dev = -1;
@@ -925,7 +947,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
         const float* kin;
         float* kout;
         if (n > 1) {
-            const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
+            const int f0 = (int)bounds[c], f1 = (int)bounds[c + 1];
             if (frames_contig) {
                 if ((err = cudaMemcpyAsync(din + f0 * plane, h_in + f0 * plane, sizeof(float) * plane * (f1 - f0),
                                            cudaMemcpyHostToDevice, up)) != cudaSuccess)
@@ -940,7 +962,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
             kin = din + f0 * plane;
             kout = dout + f0 * plane;
         } else {
-            const int r0 = (int)((long long)h * c / chunks), r1 = (int)((long long)h * (c + 1) / chunks);
+            const int r0 = (int)bounds[c], r1 = (int)bounds[c + 1];
             const int need = std::min(h, r1 + p.hy);
             if (need > copied) {
                 if ((err = cudaMemcpy2DAsync(din + (long long)copied * w, rowb, h_in + (long long)copied * img->pitch,
@@ -960,7 +982,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
         if ((err = cudaEventRecord(ev[3 * c + 1], cs)) != cudaSuccess) return bail(err, "record");
         if ((err = cudaStreamWaitEvent(down, ev[3 * c + 1], 0)) != cudaSuccess) return bail(err, "wait");
         if (n > 1) {
-            const int f0 = (int)((long long)n * c / chunks), f1 = (int)((long long)n * (c + 1) / chunks);
+            const int f0 = (int)bounds[c], f1 = (int)bounds[c + 1];
             if (frames_contig) {
                 if ((err = cudaMemcpyAsync(h_out + f0 * plane, dout + f0 * plane, sizeof(float) * plane * (f1 - f0),
                                            cudaMemcpyDeviceToHost, down)) != cudaSuccess)
@@ -972,7 +994,7 @@ paraprox_status paraprox_run_host(paraprox_filter f, paraprox_scheme scheme, int
                         return bail(err, "D2H");
             }
         } else {
-            const int r0 = (int)((long long)h * c / chunks), r1 = (int)((long long)h * (c + 1) / chunks);
+            const int r0 = (int)bounds[c], r1 = (int)bounds[c + 1];
             if ((err = cudaMemcpy2DAsync(h_out + (long long)r0 * img->pitch, sizeof(float) * img->pitch,
                                          dout + (long long)r0 * w, rowb, rowb, r1 - r0, cudaMemcpyDeviceToHost,
                                          down)) != cudaSuccess)

@@ -233,7 +233,11 @@ def test_tuner_tpins_on_gpu(P):
 
 
 def test_run_host_matches_device_path(P):
-    for shape, w in [((1, 1500, 900), F.conv(9)), ((5, 120, 256), F.mean(5))]:
+    # single-chunk shapes, then shapes that take the ramped chunk schedule
+    # (row bands of 64/128/256 rows at both ends of a 2048 x 4096 image with a
+    # 4-row halo; 1/1/2-frame chunks at both ends of a 40-frame batch)
+    for shape, w in [((1, 1500, 900), F.conv(9)), ((5, 120, 256), F.mean(5)), ((1, 2048, 4096), F.conv(9)),
+                     ((40, 256, 2048), F.mean(5))]:
         x = torch.from_numpy(W.frames(*shape, seed0=12)).pin_memory()
         f = P.Filter(w)
         for scheme, d in [("exact", 0), ("row", 1), ("center", 2)]:
