@@ -311,6 +311,9 @@ for name, w, m in [("mean5", F.mean(5), "mre"), ("conv9", F.conv(9), "l2"), ("se
     f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
     x = torch.from_numpy(W.frames(4, 160, 200, 3)).cuda()
     out[name] = P.tune_partials(x, f, m).tolist()
+    # 6144 tiles: two waves of the bounded-persistence schedule
+    xb = torch.from_numpy(W.frames(3, 4096, 4096, 5)).cuda()
+    out[name + "_waves"] = P.tune_partials(xb, f, m).tolist()
 print(json.dumps(out))
 ''' % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))),)
     res = {}
@@ -322,9 +325,45 @@ print(json.dumps(out))
     metric = {"mean5": "mre", "conv9": "l2", "sep7": "l2"}
     for name in res["1"]:
         a, b = np.array(res["1"][name]), np.array(res["0"][name])
-        qa = [P.quality_from_partials(a[3 * k:3 * k + 3], metric[name]) for k in range(len(a) // 3)]
-        qb = [P.quality_from_partials(b[3 * k:3 * k + 3], metric[name]) for k in range(len(b) // 3)]
+        mt = metric[name.split("_")[0]]
+        qa = [P.quality_from_partials(a[3 * k:3 * k + 3], mt) for k in range(len(a) // 3)]
+        qb = [P.quality_from_partials(b[3 * k:3 * k + 3], mt) for k in range(len(b) // 3)]
         np.testing.assert_allclose(qa, qb, rtol=0, atol=1e-12)
+
+
+def test_tile_schedules_bitwise():
+    """Bounded persistence (default: 16 tiles per CTA, 8 for the lattice)
+    and the fully persistent grid (PARAPROX_TILE_CHUNK=0 /
+    PARAPROX_LATTICE_CHUNK=0) compute every tile with the same code: outputs
+    are bit-identical, here on 6144 tiles (two waves) with ragged edges."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import hashlib, sys, torch
+sys.path.insert(0, %r)
+import paper_conf_asplos_samadijlm14_b200 as pkg
+import workloads as W
+from workloads import filters as F
+P = pkg.paraprox
+x = torch.from_numpy(W.frames(3, 4090, 4093, 7)).cuda()
+h = hashlib.sha256()
+for w in (F.mean(5), F.conv(9), F.gaussian(3)):
+    f = P.Filter(w)
+    for scheme, d in (("exact", 0), ("row", 1), ("center", 1), ("col", 2)):
+        h.update(P.stencil_approx(x, f, scheme, d).cpu().numpy().tobytes())
+    h.update(P.stencil_lattice(x, f, "row", 1).cpu().numpy().tobytes())
+fs = P.Filter(wy=F.separable(7)[0], wx=F.separable(7)[1])
+h.update(P.stencil_approx(x, fs, "row", 1).cpu().numpy().tobytes())
+print(h.hexdigest())
+''' % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))),)
+    digests = []
+    for chunk in ("16", "0"):
+        env = dict(os.environ, PARAPROX_TILE_CHUNK=chunk, PARAPROX_LATTICE_CHUNK="0" if chunk == "0" else "8")
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr
+        digests.append(r.stdout.strip().splitlines()[-1])
+    assert digests[0] == digests[1]
 
 
 def test_tma_store_and_register_store_epilogues_bitwise():
