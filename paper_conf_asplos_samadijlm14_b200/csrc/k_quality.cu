@@ -83,7 +83,10 @@ __global__ void __launch_bounds__(256) k_quality_flat(const float* __restrict__ 
     };
     sweep([&](float e, float a) { q.add(e, a); });
     if constexpr (M == PARAPROX_MRE)
-        if (__syncthreads_or(q.bad)) sweep([&](float e, float a) { q.fix(e, a); });
+        if (__syncthreads_or(q.bad)) {
+            q.reset();
+            sweep([&](float e, float a) { q.fix(e, a); });
+        }
     double s0, s1;
     q.get(s0, s1);
     block_sum2(s0, s1);
@@ -135,7 +138,10 @@ __global__ void __launch_bounds__(256, M == PARAPROX_MRE ? 3 : 2) k_quality_part
     };
     sweep([&](float e, float a) { q.add(e, a); });
     if constexpr (M == PARAPROX_MRE)
-        if (__syncthreads_or(q.bad)) sweep([&](float e, float a) { q.fix(e, a); });
+        if (__syncthreads_or(q.bad)) {
+            q.reset();
+            sweep([&](float e, float a) { q.fix(e, a); });
+        }
     double s0, s1;
     q.get(s0, s1);
     block_sum2(s0, s1);

@@ -21,6 +21,7 @@ template <int M>
 struct QAcc {
     double s0 = 0.0, s1 = 0.0;
     bool bad = false;                                       // never set: no fix-up pass
+    __device__ __forceinline__ void reset() {}
     __device__ __forceinline__ void fix(float, float) {}
     __device__ __forceinline__ void add(float e, float a) {
         const double de = (double)e, da = (double)a;
@@ -53,9 +54,10 @@ __device__ __forceinline__ float rcp_approx(float x) {
 template <>
 struct QAcc<PARAPROX_MRE> {
     double hi = 0.0, lo = 0.0;  // sums of the leading and trailing parts of the terms
-    bool bad = false;  // a term the pair arithmetic cannot carry was skipped
-    // the fast path skips terms with |E| tiny or huge or |A-E| huge (and the
-    // E == 0 convention, S12); a second pass adds exactly those in fp64
+    bool bad = false;  // some term the pair arithmetic cannot carry was seen
+    // the fast path needs |E| in [1e-30, 1e30] and |A-E| <= 1e30 (and E != 0,
+    // the S12 convention); a CTA that saw any other term redoes all of its
+    // terms in fp64 (fix pass), so the fast path carries no per-term select
     __device__ __forceinline__ static bool fast_ok(float ae, float dh) {
         return ae >= 1e-30f && ae <= 1e30f && fabsf(dh) <= 1e30f;
     }
@@ -63,28 +65,23 @@ struct QAcc<PARAPROX_MRE> {
         float dh, dl;
         two_sum(a, -e, dh, dl);  // A - E exactly, as dh + dl
         const float ae = fabsf(e);
-        const bool ok = fast_ok(ae, dh);
-        bad |= !ok;
-        if (dh < 0.f) {
-            dh = -dh;
-            dl = -dl;
-        }
-        // q0 + q1 = |A-E| / |E| to ~2^-46: the remainder of the first quotient
+        bad |= !fast_ok(ae, dh);
+        // q0 + q1 = (A-E) / |E| to ~2^-46: the remainder of the first quotient
         // is exact under the FMA, so the approximate reciprocal's own error is
-        // corrected by the second term
+        // corrected by the second term; the term |q0 + q1| = |q0| + q1 * sgn(q0)
+        // (|q1| << |q0|, and q0 = 0 only when A = E)
         const float rc = rcp_approx(ae);
         const float q0 = __fmul_rn(dh, rc);
         const float rem = __fadd_rn(__fmaf_rn(-q0, ae, dh), dl);
-        hi += ok ? (double)q0 : 0.0;
-        lo += ok ? (double)__fmul_rn(rem, rc) : 0.0;
+        hi += (double)fabsf(q0);
+        const float q1 = __fmul_rn(rem, rc);
+        lo += (double)__uint_as_float(__float_as_uint(q1) ^ (__float_as_uint(q0) & 0x80000000u));  // q1 * sgn(q0)
     }
+    // fix pass: every term of the CTA again, in fp64
+    __device__ __forceinline__ void reset() { hi = lo = 0.0; }
     __device__ __forceinline__ void fix(float e, float a) {
-        float dh, dl;
-        two_sum(a, -e, dh, dl);
-        if (!fast_ok(fabsf(e), dh)) {
-            const double de = (double)e, da = (double)a;
-            hi += de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
-        }
+        const double de = (double)e, da = (double)a;
+        hi += de != 0.0 ? fabs(da - de) / fabs(de) : (da == 0.0 ? 0.0 : 1.0);
     }
     __device__ __forceinline__ void get(double& a, double& b) const {
         a = hi + lo;
