@@ -23,6 +23,7 @@ for c in c1 c3 c4; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_tiles|k_pointwise|k_lattice" -c 4 -o gpurun_out/prof_$c -f python tools/prof_run.py --workload $c --schemes exact:0,center:9 --reps 1 > gpurun_out/ncu_$c.log 2>&1; echo ncu $c rc=$?
 done
 fi
+[ -z "$NO_NCU" ] && bash tools/ncu_bytes.sh
 bash tools/sanitize.sh
 # summarise the ncu captures here on the box (gpurun_out/ must stay < 64 MiB)
 for c in c1 c2 c3 c4; do
@@ -32,5 +33,6 @@ for c in c1 c2 c3 c4; do
   fi
 done
 python tools/ncu_summary.py launches gpurun_out/launches_c2.csv > gpurun_out/launches_c2.md 2>/dev/null
+python tools/ncu_summary.py bytes gpurun_out/ncu_bytes_c2.csv gpurun_out/ncu_bytes_c4.csv > gpurun_out/ncu_bytes.md 2>/dev/null
 du -sh gpurun_out
 

@@ -3,6 +3,8 @@
     python tools/ncu_summary.py launches gpurun_out/launches_c2.csv > profiles/r01_launches_c2.md
     python tools/ncu_summary.py full gpurun_out/prof_c2.ncu-rep --workload c2 \
         --traffic profiles/traffic.json > profiles/r01_ncu_full_c2.md
+    python tools/ncu_summary.py bytes gpurun_out/ncu_bytes_c2.csv gpurun_out/ncu_bytes_c4.csv \
+        > profiles/r01_ncu_bytes.md
 """
 import argparse
 import csv
@@ -38,7 +40,7 @@ SETS = {256: "s0", 896: "f1", 1984: "f2", 4064: "f3", 8176: "f4", 1344: "l2", 23
 
 def short(name):
     """ncu kernel name -> the library's kernel name (paraprox_last_kernel())."""
-    m = re.match(r"void (?:ppx::)?k_tiles<(\d+), (\d+), (\d+)u?, (\d+)u?, (\d|true|false)>", name)
+    m = re.match(r"void (?:ppx::)?k_tiles<(\d+), (\d+), (\d+)u?, (\d+)u?, (\d|true|false)(?:, (\d|true|false))?>", name)
     if m:
         sep = m.group(5) in ("1", "true")
         return f"{'sep' if sep else 'dense'}_{SETS.get(int(m.group(3)), m.group(3))}_{SETS.get(int(m.group(4)), m.group(4))}"
@@ -111,14 +113,57 @@ def full(path, workload, traffic_json):
         json.dump(d, open(traffic_json, "w"), indent=1, sort_keys=True)
 
 
+PIXELS = {"c2": 4096 * 4096, "c4": 32768 * 32768}
+
+
+def bytes_table(paths):
+    """DRAM bytes per launch (ncu --metrics dram__bytes_*) against the
+    algorithmic bytes: 8 B/px for the stencils, 4/s + 4 B/px for the row
+    lattice of stride s (only every s-th row is read)."""
+    print("# DRAM bytes: exact vs per-window approximation vs row lattice (NEXT-1)\n")
+    print("`tools/ncu_bytes.sh`: `ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum "
+          "--clock-control none` (L2 flushed before every kernel), one launch each on the bench's input. "
+          "`alg` = algorithmic bytes per pixel; `measured` = (read + write) / pixels.\n")
+    print("| workload | kernel | read MB | write MB | measured B/px | alg B/px | measured / alg | vs exact | us (cold) |")
+    print("|---|---|---:|---:|---:|---:|---:|---:|---:|")
+    for path in paths:
+        wl = re.search(r"(c\d)", os.path.basename(path)).group(1)
+        rows = list(csv.reader(open(path)))
+        hdr = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
+        h = rows[hdr]
+        ii, ki, mi, ui, vi = (h.index("ID"), h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Unit"),
+                              h.index("Metric Value"))
+        launches = {}
+        for r in rows[hdr + 1:]:
+            if len(r) <= vi:
+                continue
+            d = launches.setdefault(r[ii], {"kernel": short(r[ki])})
+            d[r[mi]] = float(r[vi].replace(",", "")) * UNIT_SCALE.get(r[ui], 1)
+        exact_b = None
+        for _, d in sorted(launches.items(), key=lambda x: int(x[0])):
+            b = d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
+            px = PIXELS[wl]
+            m = re.match(r"lattice_\w+_s(\d+)_r\d+", d["kernel"])
+            alg = 4.0 / int(m.group(1)) + 4.0 if m else 8.0
+            if exact_b is None:
+                exact_b = b
+            t = d.get("gpu__time_duration.sum", 0.0)
+            t_us = t * 1e6 if t < 1 else t / 1e3
+            print(f"| {wl} | `{d['kernel']}` | {d.get('dram__bytes_read.sum', 0) / 1e6:.1f} | "
+                  f"{d.get('dram__bytes_write.sum', 0) / 1e6:.1f} | {b / px:.3f} | {alg:.3f} | {b / px / alg:.3f} | "
+                  f"{b / exact_b:.3f} | {t_us:.1f} |")
+
+
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("kind", choices=["launches", "full"])
-    ap.add_argument("path")
+    ap.add_argument("kind", choices=["launches", "full", "bytes"])
+    ap.add_argument("path", nargs="+")
     ap.add_argument("--workload", default="c2")
     ap.add_argument("--traffic", default=None)
     a = ap.parse_args()
     if a.kind == "launches":
-        launches(a.path)
+        launches(a.path[0])
+    elif a.kind == "bytes":
+        bytes_table(a.path)
     else:
-        full(a.path, a.workload, a.traffic)
+        full(a.path[0], a.workload, a.traffic)
