@@ -176,9 +176,32 @@ def cpu_baseline(wl, kind, w, scheme, reach, budget_s=10.0, max_reps=400):
         if time.perf_counter() - t0 >= budget_s:
             break
     dt = time.perf_counter() - t0
+    # the same oracle on one core (single-thread and all-core),
+    # a 256-row band for ~2 s
+    import ctypes
+    single = None
+    try:
+        gomp = ctypes.CDLL("libgomp.so.1")
+        gomp.omp_set_num_threads(1)
+        xb = x[:256]
+        t1 = time.perf_counter()
+        n1 = 0
+        while time.perf_counter() - t1 < 2.0 and n1 < 100:
+            oracle_run(xb, kind, w, scheme, reach)
+            n1 += 1
+        single = {"value": n1 * xb.size / (time.perf_counter() - t1) / 1e6, "cores": 1,
+                  "sample": f"{n1} x 256x{wd} band"}
+        gomp.omp_set_num_threads(cores)
+    except OSError:
+        pass
+    model = None
+    try:
+        model = next(ln.split(":", 1)[1].strip() for ln in open("/proc/cpuinfo") if ln.startswith("model name"))
+    except (OSError, StopIteration):
+        pass
     return {"value": px / dt / 1e6, "unit": "Mpixel/s", "cores": cores, "kind": "oracle",
             "sample": f"{reps} x {rows}x{wd} frame(s), {scheme}:{reach}, fp64 literal per-window oracle",
-            "seconds": dt}
+            "seconds": dt, "single_thread": single, "host_cpu": model, "nproc": os.cpu_count()}
 
 
 def dist_setup():
