@@ -651,7 +651,8 @@ def main():
     if args.e2e_steps > 0 and px_step * 4 <= (8 << 30):
         hin = inputs[0].cpu().pin_memory()
         hout = torch.empty_like(hin, pin_memory=True)
-        P.run_host(hin, f, scheme, reach, out=hout)  # warm
+        for _ in range(3):  # warm (first calls fault in the pinned pages and the scratch pool)
+            P.run_host(hin, f, scheme, reach, out=hout)
         if dist:
             dist.barrier()
         torch.cuda.synchronize()
