@@ -99,16 +99,33 @@ struct TileArgs {
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
 
-template <int HY, int HX>
+// CTAs per SM an instance is built for: 2 (up to 3 stages), or 3 with 2
+// stages for the instances where the A/B measured that faster (kbench, two
+// runs: exact 5x5 +5 %, c4 rows {-3,0,3} x all columns +8 %, c4 rows/columns
+// {-4,0,4} +5 %; most other instances lose 3-7 % and the exact 9x9 15 %)
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+__host__ __device__ constexpr int tile_min_blocks() {
+    constexpr uint32_t F2 = 0x1Fu << 6, F4 = 0x1FFu << 4;
+    constexpr uint32_t L3 = (1u << 5) | (1u << 8) | (1u << 11), L4 = (1u << 4) | (1u << 8) | (1u << 12);
+    return (!SEP && ((HY == 2 && HX == 2 && MASKY == F2 && MASKX == F2) ||
+                     (HY == 3 && HX == 4 && MASKY == L3 && MASKX == F4) ||
+                     (HY == 4 && HX == 4 && MASKY == L4 && MASKX == L4)))
+               ? 3
+               : PPX_TILE_MIN_BLOCKS;
+}
+
+template <int HY, int HX, int MINB = PPX_TILE_MIN_BLOCKS>
 struct Geom {
     static constexpr int HXP = round4(HX);
     static constexpr int SW = kTW + 2 * HXP;   // staged row length (floats)
     static constexpr int SH = kTH + 2 * HY;    // staged rows
     static constexpr int STAGE_BYTES = SW * SH * 4;
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
-    // as many stages as fit two CTAs per SM (<= 110 KiB each), 2..MAX
+    // as many stages as fit MINB CTAs per SM (2: <= 110 KiB each, 2..MAX;
+    // 3: 2 stages)
     static constexpr int FIT = (110 * 1024) / STAGE_STRIDE;
-    static constexpr int STAGES = FIT < 2 ? 2 : (FIT < PPX_TILE_MAX_STAGES ? FIT : PPX_TILE_MAX_STAGES);
+    static constexpr int STAGES =
+        MINB >= 3 ? 2 : (FIT < 2 ? 2 : (FIT < PPX_TILE_MAX_STAGES ? FIT : PPX_TILE_MAX_STAGES));
     static constexpr int SMEM = STAGES * STAGE_STRIDE;
 };
 
@@ -249,10 +266,10 @@ __host__ __device__ constexpr bool odd_pairs_faster() {
 }
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
-__global__ void __launch_bounds__(kThreads, PPX_TILE_MIN_BLOCKS) k_tiles(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASKX, SEP>())) k_tiles(const __grid_constant__ CUtensorMap tmap,
                                                        const TileArgs A, const __grid_constant__ TapW W,
                                                        const __grid_constant__ CUtensorMap omap) {
-    using G = Geom<HY, HX>;
+    using G = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()>;
     constexpr int HXP = G::HXP, SW = G::SW, SH = G::SH, NV = 4 + 2 * HXP;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ uint64_t bars[G::STAGES];
@@ -609,7 +626,7 @@ TileInstance make_instance(const char* name) {
     ti.hx = HX;
     ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP, false>;
     ti.fnq = k_tiles<HY, HX, MASKY, MASKX, SEP, true>;
-    ti.smem = Geom<HY, HX>::SMEM;
+    ti.smem = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()>::SMEM;
     ti.name = name;
     return ti;
 }
