@@ -11,6 +11,7 @@
 // Rounding matches the tile kernels bit for bit: dense fmaf(w, x, 0);
 // separable fmaf(wy, fmaf(wx, x, 0), 0) (horizontal, then vertical pass).
 #include <algorithm>
+#include <cmath>
 
 #include "quality.cuh"
 
@@ -72,21 +73,21 @@ __device__ __forceinline__ float steps1(float x, float a, float w0, float w1, co
 // array, which the A/B in tools/mapbench.cu measured 13-16 % faster at 4 GiB
 // (6.9 TB/s, above cudaMemcpy's 6.66) than the grid-stride form, whose kPU
 // loads per thread land a whole grid stride (4.8 MB) apart.
-template <bool SEP>
+template <bool SEP, int PU = kPU>
 __global__ void __launch_bounds__(256) k_pointwise_flat(const float* __restrict__ in, float* __restrict__ out,
                                                         long long count, float w0, float w1, const Addend add) {
     const long long n4 = count >> 2;
-    const long long base = (long long)blockIdx.x * (256 * kPU) + threadIdx.x;
+    const long long base = (long long)blockIdx.x * (256 * PU) + threadIdx.x;
     const float4* i4 = reinterpret_cast<const float4*>(in);
     float4* o4 = reinterpret_cast<float4*>(out);
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    float4 v[kPU];
+    float4 v[PU];
 #pragma unroll
-    for (int u = 0; u < kPU; ++u)
+    for (int u = 0; u < PU; ++u)
         if (base + u * 256 < n4) v[u] = ld_stream(i4 + base + u * 256);
 #pragma unroll
-    for (int u = 0; u < kPU; ++u)
+    for (int u = 0; u < PU; ++u)
         if (base + u * 256 < n4) {
             const long long i = base + u * 256;
             const float4 r = add.p ? steps4<SEP>(v[u], __ldcs(reinterpret_cast<const float4*>(add.p) + i), w0, w1, add)
@@ -190,11 +191,42 @@ cudaError_t launch_pointwise(const Plan& p, const float* in, const View& v, floa
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     if (flat) {
-        const long long per = 256LL * kPU;
+        // float4 per thread: kPU (16 KiB per CTA), or fewer when that leaves a
+        // mostly empty last wave of CTAs (c2: 4096 CTAs = 3.5 waves of the
+        // 1184 resident; 8 KiB chunks make 6.9 waves)
+        int pu = kPU;
+        {
+            static int resident = 0;  // CTAs per GPU (SMs x 8 at 256 threads)
+            if (!resident) {
+                int dev = 0, sms = 148, occ = 8;
+                if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointwise_flat<false>, 256, 0);
+                resident = sms * std::max(1, occ);
+            }
+            double best = 0.0;
+            for (int c : {kPU, 2, 1}) {
+                const double waves = (double)((count / 4 + 256LL * c - 1) / (256LL * c)) / resident;
+                const double eff = waves / std::ceil(waves);
+                if (eff > best + 0.02) {
+                    best = eff;
+                    pu = c;
+                }
+            }
+        }
+        const long long per = 256LL * pu;
         const long long want = (count / 4 + per - 1) / per;
         cfg.gridDim = dim3((unsigned)std::max<long long>(1, std::min<long long>(want, 0x7fffffffLL)));
-        err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_flat<true>, in, out, count, w0, w1, add)
-                          : cudaLaunchKernelEx(&cfg, k_pointwise_flat<false>, in, out, count, w0, w1, add);
+#define PPX_MAP_LAUNCH(PU)                                                                                  \
+    err = p.separable ? cudaLaunchKernelEx(&cfg, k_pointwise_flat<true, PU>, in, out, count, w0, w1, add)   \
+                      : cudaLaunchKernelEx(&cfg, k_pointwise_flat<false, PU>, in, out, count, w0, w1, add);
+        if (pu == 1) {
+            PPX_MAP_LAUNCH(1)
+        } else if (pu == 2) {
+            PPX_MAP_LAUNCH(2)
+        } else {
+            PPX_MAP_LAUNCH(kPU)
+        }
+#undef PPX_MAP_LAUNCH
         count_launch(p.separable ? "sep_map" : "dense_map");
     } else {
         const long long rows = (long long)v.n * v.h;
