@@ -135,6 +135,21 @@ int oracle_hotspot(const float* temp, const float* power, int n, int h, int w,
                    double c, double gx, double gy, double gz, double tamb,
                    int dy, int dx, int iterations, double* out);
 
+/* Runtime loop (§2, §5;
+ * readings DESIGN.md R1-R4).
+ * oracle_runtime_ladder: from the m candidates' training qualities (cost
+ * order), rung 0 = the first with q >= toq, then every later candidate whose
+ * q is strictly above all earlier rungs, then EXACT (written as -1).  Writes
+ * up to cap candidate indices to rungs; returns the rung count (or -1).
+ * oracle_runtime_trace: the rung each of t_count invocations runs on, given
+ * q[t * rungs + k] = the quality a check of invocation t would measure on
+ * rung k.  Invocation t is checked when check_every > 0, t % check_every ==
+ * 0 and the rung is not EXACT (the last); a check below toq moves one rung
+ * down before invocation t + 1.  checked[t] (optional) flags the checks. */
+int oracle_runtime_ladder(int m, const double* train_q, double toq, int cap, int* rungs);
+int oracle_runtime_trace(int rungs, int check_every, double toq, int t_count, const double* q,
+                         int* rung_used, int* checked, long long* checks, long long* backoffs);
+
 #ifdef __cplusplus
 }
 #endif

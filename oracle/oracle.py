@@ -76,7 +76,10 @@ def lib():
                                         C.c_int, C.c_double, C.c_int, C.c_int, f64, i32, i32, i32, f64]
         _lib.oracle_hotspot.argtypes = [f32, f32, C.c_int, C.c_int, C.c_int, C.c_double, C.c_double, C.c_double,
                                         C.c_double, C.c_double, C.c_int, C.c_int, C.c_int, f64]
-        for name in ("oracle_hotspot", "oracle_scheme_skips", "oracle_stencil_skip", "oracle_stencil_skip_sep",
+        _lib.oracle_runtime_ladder.argtypes = [C.c_int, f64, C.c_double, C.c_int, i32]
+        _lib.oracle_runtime_trace.argtypes = [C.c_int, C.c_int, C.c_double, C.c_int, f64, i32, i32,
+                                              P(C.c_longlong), P(C.c_longlong)]
+        for name in ("oracle_runtime_ladder", "oracle_runtime_trace", "oracle_hotspot", "oracle_scheme_skips", "oracle_stencil_skip", "oracle_stencil_skip_sep",
                      "oracle_tune_candidates_ex", "oracle_tune_ex", "oracle_tune_lattice", "oracle_lattice_map", "oracle_stencil_lattice", "oracle_stencil_lattice_sep",
                      "oracle_index_map", "oracle_scheme_reaches", "oracle_stencil_exact",
                      "oracle_stencil_approx", "oracle_stencil_sep", "oracle_quality",
@@ -345,3 +348,53 @@ def hotspot(temp, power, params, dy: int = 0, dx: int = 0, iterations: int = 1) 
                              float(params["gz"]), float(params["tamb"]), int(dy), int(dx), int(iterations), _dp(out)),
         "hotspot")
     return out[0] if squeeze else out
+
+
+def runtime_ladder(train_q, toq: float):
+    """R1-R2 (oracle.h): candidate indices of the ladder's rungs, -1 = EXACT."""
+    q = np.ascontiguousarray(train_q, dtype=np.float64)
+    cap = q.size + 1
+    r = np.zeros(cap, dtype=np.int32)
+    n = lib().oracle_runtime_ladder(q.size, _dp(q), float(toq), cap, r.ctypes.data_as(C.POINTER(C.c_int)))
+    _ok(0 if n > 0 else -1, "runtime_ladder")
+    return [int(v) for v in r[:n]]
+
+
+def runtime_trace(q, check_every: int, toq: float):
+    """R3-R4 (oracle.h): q[t][k] = quality a check of invocation t measures on
+    rung k.  Returns dict(rungs=[rung used per invocation], checked=[0/1],
+    checks, backoffs)."""
+    q = np.ascontiguousarray(q, dtype=np.float64)
+    t_count, rungs = q.shape
+    used = np.zeros(max(1, t_count), dtype=np.int32)
+    chk = np.zeros(max(1, t_count), dtype=np.int32)
+    nc, nb = C.c_longlong(), C.c_longlong()
+    _ok(lib().oracle_runtime_trace(rungs, int(check_every), float(toq), t_count, _dp(q),
+                                   used.ctypes.data_as(C.POINTER(C.c_int)), chk.ctypes.data_as(C.POINTER(C.c_int)),
+                                   C.byref(nc), C.byref(nb)), "runtime_trace")
+    return dict(rungs=[int(v) for v in used[:t_count]], checked=[int(v) for v in chk[:t_count]],
+                checks=nc.value, backoffs=nb.value)
+
+
+def runtime_simulate(train, frames, w, toq: float, metric="mre", check_every: int = 1):
+    """The whole runtime loop on the oracle's own stencils: ladder from the
+    oracle tuner's training qualities, then each invocation's check quality
+    = quality(exact, approx of the rung) on that frame, both rounded to fp32
+    (what the user gets), and the back-off trace.  `w` dense 2-D or (wy, wx).
+    Returns dict(ladder=[(scheme, reach, train_q)], trace=..., q=[[...]])."""
+    sep = isinstance(w, (tuple, list))
+    ky, kx = (np.asarray(w[0]).size, np.asarray(w[1]).size) if sep else np.asarray(w).shape
+    cands = tune_candidates(ky, kx, sep)
+    tq = tune(train, w, 2.0, metric, all_qualities=True)["qualities"]
+    idx = runtime_ladder(tq, toq)
+    ladder = [(cands[k][0], cands[k][1], tq[k]) if k >= 0 else ("exact", 0, 1.0) for k in idx]
+    frames, _ = _frames(frames)
+    q = np.ones((frames.shape[0], len(ladder)))
+    for t in range(frames.shape[0]):
+        x = frames[t:t + 1]
+        run = (lambda s, r: stencil_sep_scheme(x, w[0], w[1], s, r)) if sep else \
+            (lambda s, r: stencil_approx(x, w, s, r))
+        e = run("exact", 0).astype(np.float32)
+        for k, (s, r, _) in enumerate(ladder[:-1]):
+            q[t, k] = quality(e, run(s, r).astype(np.float32), metric)
+    return dict(ladder=ladder, trace=runtime_trace(q, check_every, toq), q=q.tolist())

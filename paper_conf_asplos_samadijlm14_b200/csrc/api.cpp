@@ -577,6 +577,10 @@ paraprox_status paraprox_stencil_peer(paraprox_filter f, paraprox_scheme scheme,
     int dy, dx;
     scheme_reaches(scheme, reach, &dy, &dx);
     const Plan& p = get_plan(f, dy, dx);
+    // a neighbour thinner than the halo would be clamped at its first row,
+    // which is not the image's edge: refuse (dist.PeerStripe checks this too)
+    if ((top_rows > 0 && top_rows < p.hy) || (bot_rows > 0 && bot_rows < p.hy))
+        return fail(PARAPROX_ERR_INVALID_ARG, "neighbour rows fewer than the plan's halo h_y");
     const int ntop = std::min(top_rows, p.hy), nbot = std::min(bot_rows, p.hy);
     cudaStream_t cs = (cudaStream_t)s;
     const View v = view_of(img);

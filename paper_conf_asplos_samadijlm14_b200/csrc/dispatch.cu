@@ -40,7 +40,8 @@ struct QualityOut {
     long long rpitch, rfs;
     int metric, ref_exact;
     double* part;
-    int grid;  // written: CTAs that wrote partials
+    long long cap_pairs;  // partial pairs the scratch holds (quality_scratch_pairs)
+    int grid;             // written: CTAs that wrote partials
 };
 
 void register_r1_dense();
@@ -226,9 +227,16 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     if (A.chunk != INT_MAX) {
         const long long waves = (nt + (long long)grid * A.chunk - 1) / ((long long)grid * A.chunk);
         if (waves * grid >= (1LL << 31)) return cudaSuccess;
-        grid = (int)(waves * grid);
+        if (qo && waves * grid > qo->cap_pairs) {
+            // one partial pair per CTA: when the tiles outnumber the pixels'
+            // share of the scratch (many tiny frames, w < 8), keep the
+            // persistent grid (<= kQualityBlocks pairs, always in the scratch)
+            A.chunk = INT_MAX;
+        } else {
+            grid = (int)(waves * grid);
+        }
     }
-    if (qo) qo->grid = grid;  // one partial pair per CTA (scratch: <= count / 8192 pairs)
+    if (qo) qo->grid = grid;  // one partial pair per CTA, grid <= qo->cap_pairs
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(kThreads);
@@ -285,7 +293,8 @@ cudaError_t launch_stencil_quality(const Plan& p, const float* in, const View& v
     init_registry();
     for (Entry& e : reg()) {
         if (e.ti.sep != p.separable || e.ti.masky != p.masky || e.ti.maskx != p.maskx) continue;
-        QualityOut qo{ref, ref_pitch, ref_fstride, (int)m, ref_exact ? 1 : 0, d_scratch, 0};
+        QualityOut qo{ref, ref_pitch, ref_fstride, (int)m, ref_exact ? 1 : 0, d_scratch,
+                      (long long)quality_scratch_pairs((long long)v.n * v.h * v.w), 0};
         bool taken = false;
         // the output pointer only fixes the layout checks: nothing is stored
         cudaError_t err = launch_tiles(e, p, in, v, const_cast<float*>(ref), ref_pitch, ref_fstride, s, nullptr,

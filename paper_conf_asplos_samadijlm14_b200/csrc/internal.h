@@ -135,6 +135,8 @@ constexpr int kQualityBlocks = 1184;  // partial-count cap of the persistent (ti
 // scratch (doubles) launch_quality and launch_stencil_quality need for an
 // image of `count` pixels: one partial pair per CTA
 size_t quality_scratch_doubles(long long count);
+// partial pairs that scratch holds (a quality grid must not exceed it)
+size_t quality_scratch_pairs(long long count);
 
 // ---- api.cpp helpers shared with runtime.cpp ----
 #define PPX_CUDA(call)                                  \

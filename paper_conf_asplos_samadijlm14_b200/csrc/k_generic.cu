@@ -18,8 +18,9 @@ __global__ void __launch_bounds__(256) k_stencil_generic(const float* __restrict
                                                          long long ofs, const __grid_constant__ TapTable t,
                                                          const Addend add) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
-    const int y = blockIdx.y * blockDim.y + threadIdx.y;
-    if (x >= v.w || y >= v.h) return;
+    if (x >= v.w) return;
+    // grid-stride over rows and frames: any h, n the ABI accepts launches
+    for (int y = blockIdx.y * blockDim.y + threadIdx.y; y < v.h; y += gridDim.y * blockDim.y)
     for (int f = blockIdx.z; f < v.n; f += gridDim.z) {
         const float* F = in + (long long)f * v.fstride;
         float acc = 0.f;
@@ -57,7 +58,8 @@ cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float*
     TapTable t;
     fill_taps(p, &t);
     dim3 block(32, 8);
-    dim3 grid((v.w + 31) / 32, (v.h + 7) / 8, v.n < 65535 ? v.n : 65535);
+    const int gy = (v.h + 7) / 8;
+    dim3 grid((v.w + 31) / 32, gy < 65535 ? gy : 65535, v.n < 65535 ? v.n : 65535);
     k_stencil_generic<<<grid, block, 0, s>>>(in, v, out, opitch, ofs, t, add ? *add : Addend());
     count_launch("generic");
     return cudaGetLastError();

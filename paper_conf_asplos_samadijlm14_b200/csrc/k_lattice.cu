@@ -260,11 +260,12 @@ __global__ void __launch_bounds__(256) k_lattice_generic(const float* __restrict
                                                          long long opitch, long long ofs, int dy, int dx,
                                                          const __grid_constant__ LatTaps t) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
-    const int y = blockIdx.y * blockDim.y + threadIdx.y;
-    if (x >= v.w || y >= v.h) return;
+    if (x >= v.w) return;
     const int lasty = dy ? (2 * dy + 1) * ((v.h - 1) / (2 * dy + 1)) : v.h - 1;
     const int lastx = dx ? (2 * dx + 1) * ((v.w - 1) / (2 * dx + 1)) : v.w - 1;
     const int ry = t.ky / 2, rx = t.kx / 2;
+    // grid-stride over rows and frames: any h, n the ABI accepts launches
+    for (int y = blockIdx.y * blockDim.y + threadIdx.y; y < v.h; y += gridDim.y * blockDim.y)
     for (int f = blockIdx.z; f < v.n; f += gridDim.z) {
         const float* F = in + (long long)f * v.fstride;
         float acc = 0.f;
@@ -345,7 +346,8 @@ static cudaError_t launch_lattice_generic(const paraprox_filter_s& lf, const flo
         for (int j = 0; j < lf.kx; ++j)
             t.w[i * lf.kx + j] = lf.separable ? lf.wy[i] * lf.wx[j] : lf.w[i * lf.kx + j];
     dim3 block(32, 8);
-    dim3 grid((v.w + 31) / 32, (v.h + 7) / 8, v.n < 65535 ? v.n : 65535);
+    const int gy = (v.h + 7) / 8;
+    dim3 grid((v.w + 31) / 32, gy < 65535 ? gy : 65535, v.n < 65535 ? v.n : 65535);
     k_lattice_generic<<<grid, block, 0, s>>>(in, v, out, opitch, ofs, dy, dx, t);
     count_launch("lattice_generic");
     return cudaGetLastError();

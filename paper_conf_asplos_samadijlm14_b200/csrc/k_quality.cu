@@ -250,9 +250,13 @@ cudaError_t launch_quality_final(const double* d_scratch, int g, double count, p
     return cudaGetLastError();
 }
 
-size_t quality_scratch_doubles(long long count) {
+size_t quality_scratch_pairs(long long count) {
     const long long chunks = (count + 4095) / 4096;
-    const size_t g = (size_t)(chunks > kQualityBlocks ? chunks : kQualityBlocks);
+    return (size_t)(chunks > kQualityBlocks ? chunks : kQualityBlocks);
+}
+
+size_t quality_scratch_doubles(long long count) {
+    const size_t g = quality_scratch_pairs(count);
     return 2 * g + 2 * (g / kFold + 1);  // partial pairs + the fold level
 }
 

@@ -162,11 +162,23 @@ paraprox_status paraprox_runtime_train(paraprox_runtime rt, const float* d_train
         // timing output with the training image's layout (run_stencil shares it)
         const long long fs = img->n > 1 ? img->frame_stride : (long long)img->h * img->pitch;
         const long long need = (long long)(img->n - 1) * fs + (long long)(img->h - 1) * img->pitch + img->w;
-        void* tmp = nullptr;
-        PPX_CUDA(scratch_alloc(&tmp, sizeof(float) * need, cs));
-        cudaEvent_t e0, e1;
-        PPX_CUDA(cudaEventCreate(&e0));
-        PPX_CUDA(cudaEventCreate(&e1));
+        // scratch and events released on every return path
+        struct Guard {
+            void* tmp = nullptr;
+            cudaStream_t cs = nullptr;
+            cudaEvent_t e0 = nullptr, e1 = nullptr;
+            ~Guard() {
+                if (e0) cudaEventDestroy(e0);
+                if (e1) cudaEventDestroy(e1);
+                if (tmp) cudaFreeAsync(tmp, cs);
+            }
+        } g;
+        g.cs = cs;
+        PPX_CUDA(scratch_alloc(&g.tmp, sizeof(float) * need, cs));
+        void* tmp = g.tmp;
+        PPX_CUDA(cudaEventCreate(&g.e0));
+        PPX_CUDA(cudaEventCreate(&g.e1));
+        cudaEvent_t e0 = g.e0, e1 = g.e1;
         auto time_it = [&](int dy, int dx, double* ms) -> paraprox_status {
             float best = INFINITY;
             for (int rep = 0; rep < 4; ++rep) {
@@ -193,9 +205,6 @@ paraprox_status paraprox_runtime_train(paraprox_runtime rt, const float* d_train
             }
         }
         if (st2 == PARAPROX_OK) st2 = time_it(0, 0, &rt->time_ms[c.size()]);
-        cudaEventDestroy(e0);
-        cudaEventDestroy(e1);
-        cudaFreeAsync(tmp, cs);
         if (st2 != PARAPROX_OK) return st2;
         if (first >= 0) {
             std::vector<int> up;

@@ -115,6 +115,13 @@ def _band(buf, s: Stripe, y0: int, y1: int, top: int, bottom: int):
     return buf[c + y0 - top:c + y1 + bottom], top, bottom
 
 
+def scheme_xy(scheme, reach: int):
+    """Per-axis reaches (d_y, d_x) of a scheme (O4)."""
+    dy = {"exact": 0, "row": reach, "col": 0, "center": reach, "centre": reach}[scheme]
+    dx = {"exact": 0, "row": 0, "col": reach, "center": reach, "centre": reach}[scheme]
+    return dy, dx
+
+
 def stencil_stripe(buf: torch.Tensor, s: Stripe, f, scheme, reach: int, out: torch.Tensor,
                    group=None, compute=None, hy: int | None = None):
     """One row-stripe step: halo exchange overlapped with the interior rows,
@@ -126,9 +133,7 @@ def stencil_stripe(buf: torch.Tensor, s: Stripe, f, scheme, reach: int, out: tor
         def compute(band, ht, hb, o):
             P.stencil_approx(band, f, scheme, reach, out=o, halo_top=ht, halo_bottom=hb)
     if hy is None:
-        dy = {"exact": 0, "row": reach, "col": 0, "center": reach, "centre": reach}[scheme]
-        dx = {"exact": 0, "row": 0, "col": reach, "center": reach, "centre": reach}[scheme]
-        hy = f.plan_info(dy, dx)["halo_y"]
+        hy = f.plan_info(*scheme_xy(scheme, reach))["halo_y"]
     n = s.rows
     ht, hb = s.halo_top(hy), s.halo_bottom(hy)
     if hy == 0 or n <= 2 * hy:
@@ -237,11 +242,18 @@ class PeerStripe:
 
     def stencil(self, f, scheme, reach: int, out: torch.Tensor):
         pitch = self.top_pitch if self.top is not None else self.bot_pitch
+        hy = f.plan_info(*scheme_xy(scheme, reach))["halo_y"]
+        for rows in (self.top_rows, self.bot_rows):
+            if 0 < rows < hy:
+                raise ValueError("stripe thinner than the halo")
         return self.P.stencil_peer(self.buf, f, scheme, reach, out=out, top=self.top, top_rows=self.top_rows,
                                    bot=self.bot, bot_rows=self.bot_rows, src_pitch=pitch)
 
     def close(self):
+        # every rank's kernels that read a neighbour's buf over the mapping
+        # finish before any rank unmaps or frees
         torch.cuda.synchronize()
+        dist.barrier(group=self.group)
         for base in self._opened:
             self.P.ipc_close(base)
         self._opened = []

@@ -28,7 +28,10 @@ def dev(x):
                                            ("conv9", F.conv(9), "l2"), ("sep7", F.separable(7), "l2")])
 def test_ladder(P, O, name, w, metric):
     f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
-    train = dev(W.frames(4, 192, 256, 0))
+    x = W.frames(4, 192, 256, 0)
+    train = dev(x)
+    tq_or = O.tune(x, w, 2.0, metric, all_qualities=True)["qualities"]
+    cands_or = O.tune_candidates(f.ky, f.kx, f.separable)
     for toq in (0.80, 0.90, 0.95, 0.99):
         rt = P.Runtime(f, toq, metric, check_every=10)
         st = rt.train(train)
@@ -42,6 +45,11 @@ def test_ladder(P, O, name, w, metric):
         order = P.tune_candidates(f)
         idx = [order.index(r[:2]) for r in lad[:-1]]
         assert idx == sorted(idx)                                                 # cost order kept
+        # the oracle's ladder (R1-R2 on the oracle tuner's training qualities)
+        ref = O.runtime_ladder(tq_or, toq)
+        want = [(cands_or[k][0], cands_or[k][1]) if k >= 0 else ("exact", 0) for k in ref]
+        assert [r[:2] for r in lad] == want, (toq, lad, want)
+        np.testing.assert_allclose(qs, [tq_or[k] if k >= 0 else 1.0 for k in ref], rtol=0, atol=1e-7)
         rt.close()
 
 
@@ -150,3 +158,47 @@ def test_profiled_training_picks_the_fastest_passing(P):
     out = torch.empty_like(x)
     rt.run(x, out=out)
     assert torch.equal(out, P.stencil_approx(x, f, st["scheme"], st["reach"]))
+
+
+@pytest.mark.parametrize("name,w,metric,every", [("mean5", F.mean(5), "mre", 2), ("conv9", F.conv(9), "l2", 3),
+                                                 ("sep7", F.separable(7), "l2", 1)])
+def test_backoff_trace_matches_oracle(P, O, name, w, metric, every):
+    """R3-R4 against the oracle's model: the same invocation sequence --
+    natural frames, then checkerboards (every approximation misses the TOQ),
+    then natural frames again -- gives the same rung per invocation, the same
+    checked invocations and the same check qualities (to 1e-7: fp32 vs fp64
+    stencils on 96 x 128 frames) as oracle.runtime_simulate.  Each run is
+    followed by a sync, so every check is applied before the next invocation
+    (the oracle model's order)."""
+    f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+    train = W.frames(3, 96, 128, 0)
+    nat = W.frames(12, 96, 128, 40)
+    yy, xx = np.mgrid[0:96, 0:128]
+    board = (16.0 + 219.0 * ((yy // 1 + xx // 1) % 2)).astype(np.float32)
+    seq = np.stack([nat[0], nat[1], nat[2], nat[3], board, nat[4], nat[5], board, nat[6], board, nat[7],
+                    board, nat[8], nat[9], board, nat[10], nat[11]])
+    toq = 0.9
+    sim = O.runtime_simulate(train, seq, tuple(w) if isinstance(w, tuple) else w, toq, metric, check_every=every)
+    rt = P.Runtime(f, toq, metric, check_every=every)
+    rt.train(dev(train))
+    lad = rt.ladder()
+    assert [r[:2] for r in lad] == [r[:2] for r in sim["ladder"]]
+    out = torch.empty((1, 96, 128), device="cuda")
+    used, qs = [], []
+    for t in range(seq.shape[0]):
+        before = rt.state()
+        used.append([r[:2] for r in lad].index((before["scheme"], before["reach"])))
+        rt.run(dev(seq[t:t + 1]), out=out)
+        rt.sync()
+        after = rt.state()
+        if after["checks"] > before["checks"]:
+            qs.append((t, after["last_quality"]))
+    tr = sim["trace"]
+    assert used == tr["rungs"], (used, tr["rungs"])
+    assert [t for t, _ in qs] == [t for t, c in enumerate(tr["checked"]) if c]
+    for t, q in qs:
+        assert q == pytest.approx(sim["q"][t][tr["rungs"][t]], abs=1e-7), t
+    s = rt.state()
+    assert (s["checks"], s["backoffs"]) == (tr["checks"], tr["backoffs"])
+    assert tr["backoffs"] >= 1, "the sequence must exercise a back-off"
+    rt.close()
