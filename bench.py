@@ -13,9 +13,12 @@ L1620-1628); the exact stencil (a2) is timed the same way in the same run for
 the speedup, and the quality (a4) of the chosen configuration is measured on
 the held-out frames.  DESIGN.md "Measurement" has the details.
 
-Default workload c2 (BASELINE.json configs[1]): 4096x4096 fp32, 5x5 mean, MRE.
-Weak scaling: every rank processes its own frames; no collective on the data
-path (a barrier brackets the timed region; times are max over ranks).
+Default workload c3 (BASELINE.json configs[2], the config the metric's
+"1/2/4/8 B200" is quoted on): a batch of 256 frames 3840x2160 fp32, 7x7
+separable filter, L2 quality, frame-sharded over the ranks with no collective
+on the data path (strong scaling: the 256-frame batch is the work at every N;
+a barrier brackets the timed region; times are max over ranks).  c1, c2 and
+c4 (`--workload`) are the other configs; c4 at N > 1 runs row stripes.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
 """
@@ -217,6 +220,10 @@ def dist_setup():
         torch.cuda.set_device(local)
         backend = os.environ.get("PARAPROX_DIST_BACKEND", "nccl")
         if backend == "nccl":
+            # communicator setup on stderr (ranks, transports: NVLink P2P /
+            # NVLS), so a scaling run shows which fabric NCCL used
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
@@ -255,7 +262,8 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "Mpixel/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "higher_is_better": True, "scaling": "strong" if args.workload == "c3" else "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
         "config": {"workload": args.workload, "desc": wl["desc"], "sample_rows": band, "scheme": scheme,
                    "reach": reach, "toq": args.toq},
         "cpu_baseline": {"value": value, "unit": "Mpixel/s", "cores": cores, "kind": "oracle",
@@ -297,43 +305,62 @@ def run_stripes(args, dist, rank, ws, local):
     scheme, reach, q_train = P.tune_decide(f, pt.cpu().numpy(), args.toq, wl["metric"])
     tune_ms = 1e3 * (time.perf_counter() - t0)
     del train
-    dy, dx = {"exact": (0, 0), "row": (reach, 0), "col": (0, reach), "center": (reach, reach)}[scheme]
-    hy = f.plan_info(dy, dx)["halo_y"]
+    s95, r95, q95 = P.tune_decide(f, pt.cpu().numpy(), 0.95, wl["metric"])
+
+    def halo_y(sch, rch):
+        return f.plan_info(*D.scheme_xy(sch, rch))["halo_y"]
 
     def timed(step):
+        """Median over --reps timed regions of exactly K steps (barrier +
+        synchronize on both sides, max over ranks)."""
         for _ in range(args.warmup):
             step()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        dist.barrier()
-        torch.cuda.synchronize()
-        l0 = P.launch_count()
-        e0.record(stream)
-        for _ in range(args.steps):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        dist.barrier()
-        launches = P.launch_count() - l0
-        tot = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
-        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-        return float(tot[0]) / args.steps, launches
+        runs = []
+        for _ in range(max(1, args.reps)):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            dist.barrier()
+            torch.cuda.synchronize()
+            l0 = P.launch_count()
+            e0.record(stream)
+            for _ in range(args.steps):
+                step()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            dist.barrier()
+            launches = P.launch_count() - l0
+            tot = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
+            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+            runs.append(float(tot[0]) / args.steps)
+        return float(statistics.median(runs)), launches, runs
 
-    if args.halo == "peer":
-        # the neighbours' boundary rows are read inside the stencil kernel
-        # through CUDA IPC mappings (NVLink P2P): no collective per step
-        ps = D.PeerStripe(s, wd, dev)
-        ps.buf.copy_(buf[s.cap:s.cap + s.rows])
-        del buf
-        ps.ready()
-        step_approx = lambda: ps.stencil(f, scheme, reach, out)  # noqa: E731
-        step_exact = lambda: ps.stencil(f, "exact", 0, out)  # noqa: E731
-    else:
-        step_approx = lambda: D.stencil_stripe(buf, s, f, scheme, reach, out)  # noqa: E731
-        step_exact = lambda: D.stencil_stripe(buf, s, f, "exact", 0, out)  # noqa: E731
+    # both halo paths on the same stripes: the neighbours' boundary rows read
+    # inside the stencil kernel through CUDA IPC mappings (NVLink P2P, no
+    # collective per step), and NCCL send/recv of the h_y rows overlapped
+    # with the interior rows
+    ps = D.PeerStripe(s, wd, dev)
+    ps.buf.copy_(buf[s.cap:s.cap + s.rows])
+    ps.ready()
+    modes = {
+        "peer": lambda sch, rch: (lambda: ps.stencil(f, sch, rch, out)),
+        "nccl": lambda sch, rch: (lambda: D.stencil_stripe(buf, s, f, sch, rch, out)),
+    }
+    arms = {"toq90": (scheme, reach, q_train), "toq95": (s95, r95, q95), "exact": ("exact", 0, None)}
+    res = {}
     with ClockSampler(local) as clk:
-        ms, launches = timed(step_approx)
-        approx_kernel = P.last_kernel()
-        ex_ms, _ = timed(step_exact)
+        for mode in (args.halo, "nccl" if args.halo == "peer" else "peer"):
+            res[mode] = {}
+            for name, (sch, rch, q) in arms.items():
+                ms_, nl, runs = timed(modes[mode](sch, rch))
+                hy_ = halo_y(sch, rch)
+                res[mode][name] = {"scheme": sch, "reach": rch, "quality_train": q, "ms_per_step": ms_,
+                                   "ms_per_step_reps": runs, "kernel": P.last_kernel(), "launches": nl,
+                                   "value": h * wd / (ms_ * 1e-3) / 1e6, "halo_y": hy_,
+                                   "halo_bytes_per_step_per_neighbour": hy_ * wd * 4}
+            for name in ("toq90", "toq95"):
+                res[mode][name]["speedup_vs_exact"] = res[mode]["exact"]["ms_per_step"] / res[mode][name]["ms_per_step"]
+    head = res[args.halo]["toq90"]
+    ms, launches, approx_kernel, hy = head["ms_per_step"], head["launches"], head["kernel"], head["halo_y"]
+    ex_ms = res[args.halo]["exact"]["ms_per_step"]
     peak, peak_kind = load_peaks()
     local_bytes = 8.0 * s.rows * wd
     if rank == 0:
@@ -342,7 +369,7 @@ def run_stripes(args, dist, rank, ws, local):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "c4", "desc": wl["desc"] + ", row stripes", "h": h, "w": wd, "filter": "conv9",
-                       "toq": args.toq, "metric_quality": wl["metric"],
+                       "toq": args.toq, "metric_quality": wl["metric"], "halo": args.halo,
                        "parallelism": (f"row stripes x{ws}: {s.rows} rows per rank, h_y halo rows read in-kernel "
                                        f"from the neighbours over CUDA IPC / NVLink" if args.halo == "peer" else
                                        f"row stripes x{ws}: {s.rows} rows per rank, NCCL halo send/recv of h_y rows"),
@@ -352,6 +379,8 @@ def run_stripes(args, dist, rank, ws, local):
             "exact": {"ms_per_step": ex_ms, "value": h * wd / (ex_ms * 1e-3) / 1e6, "halo_y": r,
                       "halo_bytes_per_step_per_neighbour": r * wd * 4},
             "speedup_vs_exact": ex_ms / ms,
+            "halo_modes": res,
+            "timing": {"reps": max(1, args.reps), "reported": "median of the reps' timed regions (each exactly K steps)"},
             "roofline": {"bound": "hbm", "achieved": local_bytes / (ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
                          "frac": local_bytes / (ms * 1e-3) / 1e9 / peak, "traffic": None,
                          "kernel": approx_kernel, "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
@@ -361,8 +390,7 @@ def run_stripes(args, dist, rank, ws, local):
         }
         print(json.dumps(line), flush=True)
     dist.barrier()
-    if args.halo == "peer":
-        ps.close()
+    ps.close()
     dist.destroy_process_group()
 
 
@@ -372,7 +400,8 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="c3", choices=sorted(WORKLOADS))
+    ap.add_argument("--reps", type=int, default=5, help="timed repetitions of K steps (the median is reported)")
     ap.add_argument("--toq", type=float, default=0.90)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=40)
@@ -403,8 +432,8 @@ def main():
     # c3 (configs[2]: "batch of 256 frames ... frame-sharded across 1/2/4/8"):
     # the 256 frames are split over the ranks (strong scaling, no collective on
     # the data path); the other workloads give every rank its own batch (weak)
-    strong = args.workload == "c3" and ws > 1
-    if strong:
+    strong = args.workload == "c3"
+    if strong and ws > 1:
         from paper_conf_asplos_samadijlm14_b200 import dist as D
         f0, f1 = D.frame_shard(n, ws, rank)
         assert (f1 - f0) * ws == n, "c3 needs a rank count that divides 256"
@@ -436,11 +465,13 @@ def main():
     # ---- tune once (paper: first 10 executions train) ----------------------
     torch.cuda.synchronize()
     t0 = time.perf_counter()
+    pooled_parts = None
     if ws > 1:
         parts = P.tune_partials(train, f, wl["metric"])
         pt = torch.from_numpy(parts).to(dev)
         dist.all_reduce(pt)
-        scheme, reach, q_train = P.tune_decide(f, pt.cpu().numpy(), args.toq, wl["metric"])
+        pooled_parts = pt.cpu().numpy()
+        scheme, reach, q_train = P.tune_decide(f, pooled_parts, args.toq, wl["metric"])
     else:
         scheme, reach, q_train = P.tune(train, f, args.toq, wl["metric"])
     tune_ms = 1e3 * (time.perf_counter() - t0)  # first call: includes one-time kernel setup
@@ -462,31 +493,45 @@ def main():
     plan = f.plan_info(*{"exact": (0, 0), "row": (reach, 0), "col": (0, reach),
                          "center": (reach, reach)}[scheme])
 
-    def timed(fn, steps, warmup):
-        """K back-to-back steps between two events on the launching stream,
-        barrier + synchronize on both sides, max over ranks.  Each step is one
-        kernel launch, so the kernel's average launch duration is total / K
-        (gaps between launches included: conservative)."""
-        for k in range(warmup):
-            fn(k)
-        t_all0 = torch.cuda.Event(enable_timing=True)
-        t_all1 = torch.cuda.Event(enable_timing=True)
+    def _bracket(enqueue, steps):
+        """One timed region: barrier + synchronize, two events on the
+        launching stream around exactly `steps` steps, synchronize + barrier,
+        max over ranks.  Returns the region's ms."""
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
         if dist:
             dist.barrier()
         torch.cuda.synchronize()
-        l0 = P.launch_count()
-        t_all0.record(stream)
-        for k in range(steps):
-            fn(k)
-        t_all1.record(stream)
+        t0.record(stream)
+        enqueue(steps)
+        t1.record(stream)
         torch.cuda.synchronize()
         if dist:
             dist.barrier()
-        launches = P.launch_count() - l0
-        tot = torch.tensor([t_all0.elapsed_time(t_all1)], device=dev, dtype=torch.float64)
+        tot = torch.tensor([t0.elapsed_time(t1)], device=dev, dtype=torch.float64)
         if dist:
             dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-        return float(tot[0]), float(tot[0]) / steps, launches
+        return float(tot[0])
+
+    def _median_of(enqueue, steps, reps):
+        runs = [_bracket(enqueue, steps) for _ in range(reps)]
+        return float(statistics.median(runs)), runs
+
+    def timed(fn, steps, warmup, reps=1):
+        """K back-to-back eager steps per timed region (each step is one
+        kernel launch, so the kernel's average launch duration is total / K,
+        gaps between launches included: conservative); the median region of
+        `reps`.  Returns (total ms, ms per launch, launches per region, runs)."""
+        for k in range(warmup):
+            fn(k)
+
+        def enqueue(n):
+            for k in range(n):
+                fn(k)
+        l0 = P.launch_count()
+        tot, runs = _median_of(enqueue, steps, reps)
+        launches = (P.launch_count() - l0) // max(1, reps)
+        return tot, tot / steps, launches, runs
 
     # arguments marshalled once per buffer: the loop is one ctypes call per step
     approx_ops = [P.prepare(inputs[k], f, scheme, reach, outputs[k], stream=stream) for k in range(nbuf)]
@@ -501,8 +546,10 @@ def main():
     # CUDA graphs: the launch-bound loop (c2 kernels run ~20 us) is captured
     # once -- G launches rotating over the buffers, G a multiple of nbuf so
     # consecutive launches never reuse a buffer -- and replayed; exactly K
-    # launches run in the timed region (R replays of G plus one graph of the
-    # remainder).  The eager loop (one ctypes call per launch) is timed too.
+    # launches run in a timed region (R replays of G plus one graph of the
+    # remainder).  Every captured graph is replayed once right after capture,
+    # so no first replay (graph upload) falls in a timed region.  The eager
+    # loop (one ctypes call per launch) is timed too.
     G = nbuf * max(1, 32 // nbuf)
 
     class GraphLoop:
@@ -521,6 +568,9 @@ def main():
                         self.ops[k % nbuf]()
                 self.graphs[n] = g
             torch.cuda.synchronize()
+            for g in self.graphs.values():  # upload + first replay, untimed
+                g.replay()
+            torch.cuda.synchronize()
 
         def run(self, steps):
             r, rem = divmod(steps, G)
@@ -529,46 +579,65 @@ def main():
             if rem:
                 self.graphs[rem].replay()
 
-    def timed_graph(loop, steps, warmup):
+    def timed_graph(loop, steps, warmup, reps):
         loop.run(warmup)
-        t0 = torch.cuda.Event(enable_timing=True)
-        t1 = torch.cuda.Event(enable_timing=True)
-        if dist:
-            dist.barrier()
-        torch.cuda.synchronize()
-        t0.record(stream)
-        loop.run(steps)
-        t1.record(stream)
-        torch.cuda.synchronize()
-        if dist:
-            dist.barrier()
-        tot = torch.tensor([t0.elapsed_time(t1)], device=dev, dtype=torch.float64)
-        if dist:
-            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-        return float(tot[0]), float(tot[0]) / steps, steps  # one kernel node per step
+        tot, runs = _median_of(loop.run, steps, reps)
+        return tot, tot / steps, steps, runs  # one kernel node per step
 
     def copy_step(k):  # context: torch's own device copy of the same bytes
         outputs[k % nbuf].copy_(inputs[k % nbuf])
 
     counts = (args.steps, args.warmup)
-    if not args.no_graph:
-        approx_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, scheme, reach, outputs[k], stream=st)
-                                            for k in range(nbuf)], counts)
-        approx_kernel = P.last_kernel()
-        exact_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, "exact", 0, outputs[k], stream=st)
-                                           for k in range(nbuf)], counts)
-        exact_kernel = P.last_kernel()
+    reps = max(1, args.reps)
+
+    def make_loop(sch, rch, lattice=False):
+        return GraphLoop(lambda st: [P.prepare(inputs[k], f, sch, rch, outputs[k], stream=st, lattice=lattice)
+                                     for k in range(nbuf)], counts)
+
+    def time_arm(sch, rch, lattice=False):
+        """(total ms of K steps, ms per launch, launches, runs, kernel name):
+        graph replay by default, the eager ctypes loop with --no-graph."""
+        if args.no_graph:
+            ops = [P.prepare(inputs[k], f, sch, rch, outputs[k], stream=stream, lattice=lattice) for k in range(nbuf)]
+            tot, kern, nl, runs = timed(lambda k: ops[k % nbuf](), args.steps, args.warmup, reps)
+            return tot, kern, nl, runs, P.last_kernel()
+        loop = make_loop(sch, rch, lattice)
+        name = P.last_kernel()
+        tot, kern, nl, runs = timed_graph(loop, args.steps, args.warmup, reps)
+        return tot, kern, nl, runs, name
+
+    # the same tuner at TOQ 95 % (BASELINE configs[4] sweep point): where the
+    # tuned choice at 90 % is a map (centre, full reach), 95 % takes a tile
+    # kernel with a halo -- the non-degenerate approximation
+    toq_arms = {}
+    for label, toq_x in (("toq95", 0.95),):
+        if ws > 1:
+            sx, rx_, qx = P.tune_decide(f, pooled_parts, toq_x, wl["metric"])
+        else:
+            sx, rx_, qx = P.tune(train_keep, f, toq_x, wl["metric"])
+        toq_arms[label] = {"toq": toq_x, "scheme": sx, "reach": rx_, "quality_train": qx}
+
     with ClockSampler(local) as clk:
-        eager_total_ms, eager_kern_ms, eager_launches = timed(approx_step, args.steps, args.warmup)
+        eager_total_ms, eager_kern_ms, eager_launches, eager_runs = timed(approx_step, args.steps, args.warmup, reps)
         if args.no_graph:
             approx_kernel = P.last_kernel()
-            total_ms, kern_ms, launches = eager_total_ms, eager_kern_ms, eager_launches
-            exact_total_ms, exact_kern_ms, _ = timed(exact_step, args.steps, args.warmup)
-            exact_kernel = P.last_kernel()
+            total_ms, kern_ms, launches, runs = eager_total_ms, eager_kern_ms, eager_launches, eager_runs
         else:
-            total_ms, kern_ms, launches = timed_graph(approx_loop, args.steps, args.warmup)
-            exact_total_ms, exact_kern_ms, _ = timed_graph(exact_loop, args.steps, args.warmup)
-        copy_ms, _, _ = timed(copy_step, args.steps, args.warmup)
+            total_ms, kern_ms, launches, runs, approx_kernel = time_arm(scheme, reach)
+        exact_total_ms, exact_kern_ms, _, exact_runs, exact_kernel = time_arm("exact", 0)
+        copy_ms, _, _, _ = timed(copy_step, args.steps, args.warmup)
+
+        for label, arm in toq_arms.items():
+            if arm["scheme"] == "exact":
+                t_tot, t_kern, t_kernel = exact_total_ms, exact_kern_ms, exact_kernel
+            elif (arm["scheme"], arm["reach"]) == (scheme, reach):
+                t_tot, t_kern, t_kernel = total_ms, kern_ms, approx_kernel
+            else:
+                t_tot, t_kern, _, _, t_kernel = time_arm(arm["scheme"], arm["reach"])
+            arm.update({"kernel": t_kernel, "ms_per_step": t_tot / args.steps,
+                        "value": px_step * ws / (t_tot / args.steps * 1e-3) / 1e6, "unit": "Mpixel/s",
+                        "achieved_gbs": 8.0 * px_step / (t_kern * 1e-3) / 1e9,
+                        "speedup_vs_exact": exact_total_ms / t_tot})
 
         # a4: the quality reduction alone (exact vs approx buffers, 8 B/px read)
         qpart = torch.empty(3, dtype=torch.float64, device=dev)
@@ -578,7 +647,7 @@ def main():
 
         # eager: its per-call scratch (cudaMallocAsync) would become graph
         # memory nodes, measured slower on replay (c2: 36.6 vs 26.5 us)
-        qual_ms, qual_kern_ms, _ = timed(quality_step, args.steps, args.warmup)
+        qual_ms, qual_kern_ms, _, _ = timed(quality_step, args.steps, args.warmup)
 
         # NEXT-1: the global-lattice reading (only every (2d+1)-th row is read
         # from HBM), tuned by its own tuner at the same TOQ on the same frames
@@ -592,17 +661,10 @@ def main():
                 l_scheme, l_reach, l_q = P.tune_lattice(train_keep, f, args.toq, wl["metric"])
             lat = {"scheme": l_scheme, "reach": l_reach, "quality_train": l_q}
             if l_scheme != "exact":
-                if args.no_graph:
-                    lat_ops = [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=stream, lattice=True)
-                               for k in range(nbuf)]
-                    lat_total, lat_kern, _ = timed(lambda k: lat_ops[k % nbuf](), args.steps, args.warmup)
-                else:
-                    lat_loop = GraphLoop(lambda st: [P.prepare(inputs[k], f, l_scheme, l_reach, outputs[k], stream=st,
-                                                               lattice=True) for k in range(nbuf)], counts)
-                    lat_total, lat_kern, _ = timed_graph(lat_loop, args.steps, args.warmup)
+                lat_total, lat_kern, _, _, lat_kernel = time_arm(l_scheme, l_reach, lattice=True)
                 lat_bpp = 4.0 / (2 * l_reach + 1) + 4.0
                 lat.update({
-                    "kernel": P.last_kernel(), "ms_per_step": lat_total / args.steps,
+                    "kernel": lat_kernel, "ms_per_step": lat_total / args.steps,
                     "value": px_step * ws / (lat_total / args.steps * 1e-3) / 1e6, "unit": "Mpixel/s",
                     "algorithmic_bytes_per_px": lat_bpp,
                     "achieved_gbs": lat_bpp * px_step / (lat_kern * 1e-3) / 1e9,
@@ -641,7 +703,13 @@ def main():
         rel = np.abs(an - en) / np.maximum(np.abs(en), 1e-30)
         fig13 = {"lt_10pct": float(np.mean(rel < 0.10)), "lt_1pct": float(np.mean(rel < 0.01)),
                  "p50": float(np.median(rel)), "p99": float(np.quantile(rel, 0.99)), "pixels": int(k)}
-        del e, a, en, an, rel
+        del a, en, an, rel
+        for arm in toq_arms.values():
+            if arm["scheme"] != "exact":
+                a = P.stencil_approx(inputs[0], f, arm["scheme"], arm["reach"])
+                arm["quality_heldout"] = P.quality(e, a, wl["metric"])
+                del a
+        del e
     # Fig. 5 statistic of the timed input: share of pixels within
     # 10 % of their 8 neighbours (the inputs are calibrated to 77.5 %)
     fig5 = float(W.fig5_statistic(inputs[0][0, :min(h, 2048), :min(wd, 2048)].cpu().numpy()))
@@ -743,7 +811,13 @@ def main():
             "copy_same_bytes_gbs": alg_bytes * args.steps / (copy_ms * 1e-3) / 1e9,
             "speedup_vs_exact": exact_ms_step / ms_step,
             "launch_mode": "eager" if args.no_graph else f"cuda_graph ({G} launches per graph, replayed)",
+            "timing": {"reps": reps, "reported": "median of the reps' timed regions (each exactly K steps)",
+                       "ms_per_step_reps": [r / args.steps for r in runs],
+                       "exact_ms_per_step_reps": [r / args.steps for r in exact_runs],
+                       "eager_ms_per_step_reps": [r / args.steps for r in eager_runs]},
             "eager_ms_per_step": eager_total_ms / args.steps,
+            "graph_vs_eager": (total_ms / eager_total_ms) if not args.no_graph else 1.0,
+            "toq_arms": {k: dict(v, roofline_frac=v["achieved_gbs"] / peak) for k, v in toq_arms.items()},
             "quality_kernel": {"metric": wl["metric"], "ms": qual_kern_ms, "kernel": "quality_flat",
                                "achieved_gbs": alg_bytes / (qual_kern_ms * 1e-3) / 1e9,
                                "frac": alg_bytes / (qual_kern_ms * 1e-3) / 1e9 / peak,

@@ -1,25 +1,43 @@
 // k_hotspot.cu -- temporally blocked HotSpot steps (NEXT-4).
 //
 // HotSpot is a Stencil-Partition application (Table 1): the
-// grid is partitioned into tiles that are advanced independently.  Here one
-// CTA advances a 32 x 128 output tile by S <= 8 time steps from a single HBM
-// read: it stages T and P with an S-cell halo (clamped at the image edges) in
-// shared memory and computes step k over the tile grown by (S - k) cells of
-// halo, ping-ponging two shared buffers; cells outside the image are reset to
-// their clamped in-image cell after every step, so every step sees exactly the
-// clamp-to-edge borders of a single step (reading S7).  HBM traffic: 12 bytes
-// per output pixel per S steps instead of per step.
+// grid is partitioned into tiles that are advanced independently.  One CTA
+// advances a tile by S <= 8 time steps from a single HBM read of T and P.
 //
-// The approximation shrinks the halo: the folded 3x3 plan's accessed offsets
-// (row scheme: rows {0}; column: columns {0}) set HY / HX, so the row scheme
-// stages no halo rows at all.  Each step adds the taps in the order of the
-// tile kernels (rows ascending, columns ascending, fmaf from 0), then
-// fmaf(alpha, P, .) + beta: bit-identical to S single steps.
+// Layout: a 48 x 128 box of cells (the tile plus an 8-cell halo on the
+// accessed axes: 32 x 112 outputs for the exact stencil, 48 x 128 for the
+// row scheme, which reads no neighbour row) is held in REGISTERS: warp w owns
+// box rows 6w..6w+5, lane l columns 4l..4l+3 (T and P, 48 floats per
+// thread).  A step needs only
+//  * the west / east neighbours: the adjacent lanes' edge columns (shuffles),
+//  * the rows directly above / below a warp's six rows: the neighbouring
+//    warps publish their first and last rows in a ping-pong shared buffer
+//    (16 KB), one barrier per step.
+// The box edge has no neighbours: those cells turn to garbage one cell per
+// step, which never reaches the outputs (8 halo cells >= S steps).  Clamp to
+// the image edge (reading S7) is applied at read time in border tiles only:
+// a cell on the first / last valid row or column reads itself in place of
+// the missing neighbour, so out-of-image cells are never read by in-image
+// ones and need no fix-up between steps.
+//
+// Each step adds the taps in the order of the tile kernels (rows ascending,
+// columns ascending, fmaf from 0), then fmaf(alpha, P, .) + beta: bit-
+// identical to S single steps.  The approximation shrinks the halo: the row
+// scheme (rows {0}) stages no halo rows, needs no shared memory and no
+// barrier; the column scheme (columns {0}) no shuffles.
+//
+// The first version staged T and P in shared memory with one dependent
+// global load per staged row and thread and walked columns with a register
+// window: 182 us per step at 8192^2, 1.5x slower than one plain pass per step.
 #include "internal.h"
 
 namespace ppx {
 
-constexpr int kHsTH = 32, kHsTW = 128, kHsMaxS = 8;
+constexpr int kHsBH = 48, kHsBW = 128, kHsWarps = 8, kHsRPW = kHsBH / kHsWarps, kHsMaxS = 8;
+constexpr int kHsThreads = 32 * kHsWarps;
+#ifndef PPX_HS_MINB
+#define PPX_HS_MINB 3  // CTAs per SM the register budget is sized for
+#endif
 
 struct HsArgs {
     int n, h, w;
@@ -31,6 +49,7 @@ struct HsArgs {
     float w9[3][3];       // folded taps at [a + 1][b + 1] (0 where not accessed)
     float alpha, beta;
     int tiles_x, tiles_y;
+    int vec;  // 16-byte aligned rows everywhere: 128-bit loads and stores
     // optional peer halos (HotSpot row stripes): the ntop rows directly above
     // row 0 (T and P) and the nbot rows below row h-1, read from neighbour
     // buffers (CUDA IPC / NVLink); 0 rows = the image edge (clamp)
@@ -41,127 +60,163 @@ struct HsArgs {
 
 template <int HY, int HX>
 struct HsGeom {
-    static constexpr int RH = kHsTH + 2 * kHsMaxS * HY;  // staged rows (max halo)
-    static constexpr int RW = kHsTW + 2 * kHsMaxS * HX;  // staged columns = threads per row group
-    static constexpr int THREADS = 2 * RW;               // two row groups
-    static constexpr int SMEM = 3 * RH * RW * (int)sizeof(float);
+    static constexpr int OH = kHsBH - 2 * kHsMaxS * HY;  // output rows per tile
+    static constexpr int OW = kHsBW - 2 * kHsMaxS * HX;  // output columns per tile
+    static constexpr int SMEM = HY ? 2 * kHsWarps * 2 * kHsBW * (int)sizeof(float) : 0;
 };
 
-// Each thread owns one column of the step's region and half of its rows, and
-// walks down them with a 3 x (2HX+1) register window: 2HX+1 shared loads of
-// T, one of P and one store per cell and step.
-template <int HY, int HX>
-__global__ void __launch_bounds__(HsGeom<HY, HX>::THREADS, 2) k_hotspot_tb(const __grid_constant__ HsArgs A) {
-    using G = HsGeom<HY, HX>;
-    constexpr int RW = G::RW;
-    extern __shared__ __align__(16) float sm[];
-    float* bufP = sm + 2 * G::RH * RW;  // T ping-pongs between sm and sm + RH * RW
+__device__ __forceinline__ float hs_get(const float4& v, int c) {
+    return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+__device__ __forceinline__ void hs_set(float4& v, int c, float x) {
+    if (c == 0) v.x = x;
+    else if (c == 1) v.y = x;
+    else if (c == 2) v.z = x;
+    else v.w = x;
+}
 
+// the S steps on the registers; EDGE: the box touches a valid-row or image-
+// column edge (clamped neighbour reads), else the plain interior form
+template <int HY, int HX, bool EDGE>
+__device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[kHsRPW], const HsArgs& A,
+                                       float* bnd, int wi, int lane, int oy, int ox, int lo, int hi) {
     const int S = A.steps;
-    const int hy = S * HY, hx = S * HX;  // halo actually used by this launch
-    const int SH = kHsTH + 2 * hy, SW = kHsTW + 2 * hx;
-    int t = blockIdx.x;
-    const int f = t / (A.tiles_x * A.tiles_y);
-    t -= f * A.tiles_x * A.tiles_y;
-    const int y0 = (t / A.tiles_x) * kHsTH, x0 = (t % A.tiles_x) * kHsTW;
-    const int oy = y0 - hy, ox = x0 - hx;  // global coordinates of staged cell (0, 0)
-    const float* T = A.t + (long long)f * A.fs;
-    const float* Pw = A.p + (long long)f * A.fs;
-    const int lo = -A.ntop, hi = A.h - 1 + A.nbot;  // valid rows (peer halo rows included)
-    const bool border = oy < lo || ox < 0 || oy + SH > hi + 1 || ox + SW > A.w;
-
-    // stage T and P over the tile + halo, clamped to the valid rows and the
-    // image columns (rows of the staged box are spread over the threads,
-    // columns over the lanes); rows beyond the stripe come from the peers
-    for (int r = threadIdx.x / RW; r < SH; r += G::THREADS / RW) {
-        const int c = threadIdx.x % RW;
-        if (c < SW) {
-            const int gy = min(max(oy + r, lo), hi), gx = min(max(ox + c, 0), A.w - 1);
-            const float *srcT, *srcP;
-            if (gy < 0) {
-                const long long g = (long long)(A.ntop + gy) * A.ppitch + gx;
-                srcT = A.ptop_t + g;
-                srcP = A.ptop_p + g;
-            } else if (gy >= A.h) {
-                const long long g = (long long)(gy - A.h) * A.ppitch + gx;
-                srcT = A.pbot_t + g;
-                srcP = A.pbot_p + g;
-            } else {
-                const long long g = (long long)gy * A.pitch + gx;
-                srcT = T + g;
-                srcP = Pw + g;
-            }
-            sm[r * RW + c] = *srcT;
-            bufP[r * RW + c] = *srcP;
-        }
+    // per-row / per-column edge flags (EDGE only)
+    bool top[kHsRPW], bot[kHsRPW], wst[4], est[4];
+#pragma unroll
+    for (int i = 0; i < kHsRPW; ++i) {
+        const int gy = oy + wi * kHsRPW + i;
+        top[i] = EDGE && gy == lo;
+        bot[i] = EDGE && gy == hi;
     }
-    __syncthreads();
-
-    const int col = threadIdx.x % RW, grp = threadIdx.x / RW;
-    for (int k = 1; k <= S; ++k) {
-        const float* cur = sm + ((k - 1) & 1) * (G::RH * RW);
-        float* nxt = sm + (k & 1) * (G::RH * RW);
-        // region of step k: the tile grown by (S - k) halo cells
-        const int gyk = (S - k) * HY, gxk = (S - k) * HX;
-        const int r0 = hy - gyk, c0 = hx - gxk;
-        const int nr = kHsTH + 2 * gyk, nc = kHsTW + 2 * gxk;
-        const bool last = k == S;
-        const int c = c0 + col;
-        if (col < nc) {
-            const int half = (nr + 1) / 2;
-            const int rs = r0 + grp * half, re = min(r0 + nr, rs + half);
-            float win[3][2 * HX + 1];  // rows r-1, r, r+1 of columns c-HX..c+HX
-            if (rs < re) {
 #pragma unroll
-                for (int a = -HY; a <= 0; ++a)
+    for (int c = 0; c < 4; ++c) {
+        const int gx = ox + 4 * lane + c;
+        wst[c] = EDGE && gx == 0;
+        est[c] = EDGE && gx == A.w - 1;
+    }
+    for (int k = 0; k < S; ++k) {
+        float4 up = T[0], dn = T[kHsRPW - 1];
+        if constexpr (HY > 0) {
+            float4* B = reinterpret_cast<float4*>(bnd + (k & 1) * (kHsWarps * 2 * kHsBW));
+            B[(2 * wi) * (kHsBW / 4) + lane] = T[0];
+            B[(2 * wi + 1) * (kHsBW / 4) + lane] = T[kHsRPW - 1];
+            __syncthreads();
+            if (wi > 0) up = B[(2 * wi - 1) * (kHsBW / 4) + lane];
+            if (wi < kHsWarps - 1) dn = B[(2 * wi + 2) * (kHsBW / 4) + lane];
+        }
+        float4 prev = up;  // old value of the row above
 #pragma unroll
-                    for (int b = -HX; b <= HX; ++b) win[a + 1][b + HX] = cur[(rs + a) * RW + c + b];
+        for (int i = 0; i < kHsRPW; ++i) {
+            const float4 cur = T[i];
+            const float4 nrt = (HY && top[i]) ? cur : prev;
+            const float4 sth = (HY && bot[i]) ? cur : (i + 1 < kHsRPW ? T[i + 1] : dn);
+            float wl = 0.f, er = 0.f;
+            if constexpr (HX > 0) {
+                wl = __shfl_up_sync(0xffffffffu, cur.w, 1);
+                er = __shfl_down_sync(0xffffffffu, cur.x, 1);
             }
-#pragma unroll 4
-            for (int r = rs; r < re; ++r) {
-                if (HY) {
+            float4 nv;
 #pragma unroll
-                    for (int b = -HX; b <= HX; ++b) win[2][b + HX] = cur[(r + 1) * RW + c + b];
-                }
-                // the 5-point HotSpot taps in the tile kernels' order (N, W, C, E, S);
-                // the corners of the 3x3 are zero, and fmaf(0, x, acc) == acc
+            for (int c = 0; c < 4; ++c) {
+                const float x = hs_get(cur, c);
                 float acc = 0.f;
+                bool first = true;
 #pragma unroll
                 for (int a = -HY; a <= HY; ++a)
 #pragma unroll
-                    for (int b = -HX; b <= HX; ++b)
-                        if (a == 0 || b == 0) acc = __fmaf_rn(A.w9[a + 1][b + 1], win[a + 1][b + HX], acc);
-                acc = __fadd_rn(__fmaf_rn(A.alpha, bufP[r * RW + c], acc), A.beta);
-                if (last) {
-                    const int gy = oy + r, gx = ox + c;
-                    if (gy < A.h && gx < A.w)
-                        __stcs(A.out + (long long)f * A.fs + (long long)gy * A.pitch + gx, acc);
-                } else {
-                    nxt[r * RW + c] = acc;
-                }
-                if (HY) {
-#pragma unroll
-                    for (int b = 0; b < 2 * HX + 1; ++b) {
-                        win[0][b] = win[1][b];
-                        win[1][b] = win[2][b];
+                    for (int b = -HX; b <= HX; ++b) {
+                        if (a != 0 && b != 0) continue;
+                        float v;
+                        if (a < 0) v = hs_get(nrt, c);
+                        else if (a > 0) v = hs_get(sth, c);
+                        else if (b < 0) v = wst[c] ? x : (c == 0 ? wl : hs_get(cur, c - 1));
+                        else if (b > 0) v = est[c] ? x : (c == 3 ? er : hs_get(cur, c + 1));
+                        else v = x;
+                        acc = __fmaf_rn(A.w9[a + 1][b + 1], v, first ? 0.f : acc);
+                        first = false;
                     }
-                } else if (r + 1 < re) {
-#pragma unroll
-                    for (int b = -HX; b <= HX; ++b) win[1][b + HX] = cur[(r + 1) * RW + c + b];
-                }
+                hs_set(nv, c, __fadd_rn(__fmaf_rn(A.alpha, hs_get(Pv[i], c), acc), A.beta));
             }
+            prev = cur;
+            T[i] = nv;
         }
-        if (last) break;
-        __syncthreads();
-        // clamp-to-edge for the next step: out-of-image cells copy their edge cell
-        if (border) {
-            for (int idx = threadIdx.x; idx < nr * nc; idx += G::THREADS) {
-                const int r = r0 + idx / nc, cc = c0 + idx % nc;
-                const int gy = oy + r, gx = ox + cc;
-                const int cy = min(max(gy, lo), hi), cx = min(max(gx, 0), A.w - 1);
-                if (cy != gy || cx != gx) nxt[r * RW + cc] = nxt[(cy - oy) * RW + (cx - ox)];
+    }
+}
+
+template <int HY, int HX>
+__global__ void __launch_bounds__(kHsThreads, PPX_HS_MINB) k_hotspot_tb(const __grid_constant__ HsArgs A) {
+    using G = HsGeom<HY, HX>;
+    extern __shared__ __align__(16) float bnd[];
+    const int wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int t = blockIdx.x;
+    const int f = t / (A.tiles_x * A.tiles_y);
+    t -= f * A.tiles_x * A.tiles_y;
+    const int y0 = (t / A.tiles_x) * G::OH, x0 = (t % A.tiles_x) * G::OW;
+    const int oy = y0 - kHsMaxS * HY, ox = x0 - kHsMaxS * HX;  // global coordinates of box cell (0, 0)
+    const int lo = -A.ntop, hi = A.h - 1 + A.nbot;           // valid rows (peer halo rows included)
+    const float* Tf = A.t + (long long)f * A.fs;
+    const float* Pf = A.p + (long long)f * A.fs;
+
+    // stage: every load of the thread's 6 x 4 cells of T and P in flight at
+    // once; cells outside the valid rows / image columns read as 0 (never
+    // used by an in-image cell)
+    float4 T[kHsRPW], Pv[kHsRPW];
+    const int gx = ox + 4 * lane;
+    const bool vec_ok = A.vec && gx >= 0 && gx + 3 < A.w;
+#pragma unroll
+    for (int i = 0; i < kHsRPW; ++i) {
+        const int gy = oy + wi * kHsRPW + i;
+        T[i] = Pv[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (gy < lo || gy > hi) continue;
+        const float *ts, *ps;
+        if (gy < 0) {
+            const long long g = (long long)(A.ntop + gy) * A.ppitch;
+            ts = A.ptop_t + g;
+            ps = A.ptop_p + g;
+        } else if (gy >= A.h) {
+            const long long g = (long long)(gy - A.h) * A.ppitch;
+            ts = A.pbot_t + g;
+            ps = A.pbot_p + g;
+        } else {
+            const long long g = (long long)gy * A.pitch;
+            ts = Tf + g;
+            ps = Pf + g;
+        }
+        if (vec_ok) {
+            T[i] = __ldcs(reinterpret_cast<const float4*>(ts + gx));
+            Pv[i] = __ldg(reinterpret_cast<const float4*>(ps + gx));
+        } else {
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                if (gx + c >= 0 && gx + c < A.w) {
+                    hs_set(T[i], c, ts[gx + c]);
+                    hs_set(Pv[i], c, ps[gx + c]);
+                }
+        }
+    }
+
+    const bool edge = oy <= lo || oy + kHsBH - 1 >= hi || ox <= 0 || ox + kHsBW - 1 >= A.w - 1;
+    if (edge) hs_run<HY, HX, true>(T, Pv, A, bnd, wi, lane, oy, ox, lo, hi);
+    else hs_run<HY, HX, false>(T, Pv, A, bnd, wi, lane, oy, ox, lo, hi);
+
+    // the tile's outputs: box rows [8 HY, 8 HY + OH), columns [8 HX, 8 HX + OW)
+    float* Of = A.out + (long long)f * A.fs;
+#pragma unroll
+    for (int i = 0; i < kHsRPW; ++i) {
+        const int r = wi * kHsRPW + i;
+        const int gy = oy + r;
+        if (r < kHsMaxS * HY || r >= kHsMaxS * HY + G::OH || gy < 0 || gy >= A.h) continue;
+        float* o = Of + (long long)gy * A.pitch;
+        if (vec_ok && 4 * lane >= kHsMaxS * HX && 4 * lane + 3 < kHsMaxS * HX + G::OW) {
+            __stcs(reinterpret_cast<float4*>(o + gx), T[i]);
+        } else {
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const int bc = 4 * lane + c;
+                if (bc >= kHsMaxS * HX && bc < kHsMaxS * HX + G::OW && gx + c >= 0 && gx + c < A.w)
+                    __stcs(o + gx + c, hs_get(T[i], c));
             }
-            __syncthreads();
         }
     }
 }
@@ -200,21 +255,26 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
         A.nbot = peer->nbot;
         A.ppitch = peer->pitch;
     }
-    A.tiles_x = (v.w + kHsTW - 1) / kHsTW;
-    A.tiles_y = (v.h + kHsTH - 1) / kHsTH;
+    const auto al = [](const void* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; };
+    A.vec = al(t) && al(pw) && al(out) && (v.pitch & 3) == 0 && (v.n == 1 || (fs & 3) == 0) &&
+            (!peer || ((peer->pitch & 3) == 0 && al(peer->top_t) && al(peer->top_p) && al(peer->bot_t) &&
+                       al(peer->bot_p)));
+    const int oh = p.hy ? HsGeom<1, 0>::OH : HsGeom<0, 0>::OH, ow = p.hx ? HsGeom<0, 1>::OW : HsGeom<0, 0>::OW;
+    A.tiles_x = (v.w + ow - 1) / ow;
+    A.tiles_y = (v.h + oh - 1) / oh;
     const long long nt = (long long)A.tiles_x * A.tiles_y * v.n;
     if (nt >= (1LL << 31)) return cudaErrorInvalidValue;
-    auto launch = [&](auto kern, int smem, int threads) {
+    auto launch = [&](auto kern, int smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
-        kern<<<(unsigned)nt, threads, smem, s>>>(A);
+        kern<<<(unsigned)nt, kHsThreads, smem, s>>>(A);
         return cudaGetLastError();
     };
     cudaError_t e;
-    if (p.hy && p.hx) e = launch(k_hotspot_tb<1, 1>, HsGeom<1, 1>::SMEM, HsGeom<1, 1>::THREADS);
-    else if (p.hy) e = launch(k_hotspot_tb<1, 0>, HsGeom<1, 0>::SMEM, HsGeom<1, 0>::THREADS);
-    else if (p.hx) e = launch(k_hotspot_tb<0, 1>, HsGeom<0, 1>::SMEM, HsGeom<0, 1>::THREADS);
-    else e = launch(k_hotspot_tb<0, 0>, HsGeom<0, 0>::SMEM, HsGeom<0, 0>::THREADS);
+    if (p.hy && p.hx) e = launch(k_hotspot_tb<1, 1>, HsGeom<1, 1>::SMEM);
+    else if (p.hy) e = launch(k_hotspot_tb<1, 0>, HsGeom<1, 0>::SMEM);
+    else if (p.hx) e = launch(k_hotspot_tb<0, 1>, HsGeom<0, 1>::SMEM);
+    else e = launch(k_hotspot_tb<0, 0>, HsGeom<0, 0>::SMEM);
     if (e != cudaSuccess) return e;
     count_launch(p.hy && p.hx ? "hotspot_tb_f1_f1" : p.hy ? "hotspot_tb_f1_s0" : p.hx ? "hotspot_tb_s0_f1"
                                                                                         : "hotspot_tb_s0_s0");

@@ -20,12 +20,14 @@ final CTA.  Three comparisons per workload:
 3. `paraprox_quality` (the unfused a4 kernel) vs `oracle.quality` on the same
    stored outputs within 1e-12.
 
-QTOL: the GPU stencil sums taps in fp32, the oracle in fp64 rounded to fp32;
-per pixel the two outputs differ by a few ulps (<= 1e-6 relative, S18), with
-signs that average out over 3.4e7-1.7e8 pixels.  SURVEY 8(c) measured the
-resulting quality differences at 1e-10 - 2e-9 on 256^2 training sets; at
-these sizes they are smaller still, so QTOL = 1e-9 (the decision can flip
-only when |q - TOQ| < QTOL; the minimum margin is printed)."""
+QTOL: the two sides do not compute the same fp32 outputs.  The GPU applies
+the plan's folded weights w' = fp32(sum of the substituted taps), each
+rounded once (relative error <= 2^-24, the same sign at every pixel, so it
+does not average out), and sums taps in fp32; the oracle substitutes
+literally in fp64 and rounds the output once.  Measured on these training
+sets (r02): 1.3e-9 (c2), 2.6e-9 (c3), 1.9e-9 (c4), in line with SURVEY
+8(c)'s 1e-10 - 2e-9 at 256^2.  QTOL = 1e-8 bounds that with margin; a
+decision can flip only when |q - TOQ| < QTOL; the minimum margin is printed)."""
 import numpy as np
 import pytest
 import torch
@@ -35,7 +37,7 @@ from workloads import filters as F
 
 pytestmark = pytest.mark.gpu
 
-QTOL = 1e-9
+QTOL = 1e-8
 RTOL_REDUCTION = 1e-12
 TOQS = (0.80, 0.90, 0.95, 0.99)
 

@@ -411,7 +411,8 @@ def test_fused_quality_many_tiny_frames(P, O):
     the scratch's partial pairs (sized from the pixel count, 1250 here) under
     the bounded-persistence schedule; the fused-quality launch keeps the
     persistent grid instead.  Qualities equal the oracle's on the GPU's own
-    outputs to rounding, and the tuner's to QTOL."""
+    outputs to rounding, and the tuner's to 1e-8 (test_fullsize_tuner_gpu:
+    the folded weights are rounded to fp32 once, a bias shared by all pixels)."""
     rng = np.random.default_rng(31)
     base = W.image(160, 2000, 3)  # smooth seeded field cut into 16x16 frames
     x = np.ascontiguousarray(base.reshape(10, 16, 125, 16).transpose(0, 2, 1, 3).reshape(1250, 16, 16))
@@ -422,7 +423,7 @@ def test_fused_quality_many_tiny_frames(P, O):
     parts = P.tune_partials(xd, f, "mre")
     qg = [P.quality_from_partials(parts[3 * k:3 * k + 3], "mre") for k in range(len(cands))]
     qo = O.tune(x, F.mean(5), 2.0, "mre", all_qualities=True)["qualities"]
-    np.testing.assert_allclose(qg, qo, rtol=0, atol=1e-9)
+    np.testing.assert_allclose(qg, qo, rtol=0, atol=1e-8)
     en = P.stencil_exact(xd, f).cpu().numpy()
     for k, (s, r) in enumerate(cands):
         an = P.stencil_approx(xd, f, s, r).cpu().numpy()

@@ -58,6 +58,16 @@ def main():
         for scheme, reach in (("exact", 0), ("row", 1), ("col", 1), ("center", 1)):
             ms = graph_ms(lambda: P.hotspot(td, pd, H.PARAMS, scheme, reach, iters, out=out))
             kern = P.last_kernel()
+            # unblocked: one paraprox_hotspot call (one tile-kernel pass) per step
+            bufs = (out, torch.empty_like(td))
+
+            def per_step():
+                src = td
+                for k in range(iters):
+                    P.hotspot(src, pd, H.PARAMS, scheme, reach, 1, out=bufs[k % 2])
+                    src = bufs[k % 2]
+            ms1 = graph_ms(per_step)
+            kern1 = P.last_kernel()
             q = 1.0 if scheme == "exact" else P.quality(exact, P.hotspot(td, pd, H.PARAMS, scheme, reach, iters), "mre")
             px = td.numel()
             passes = 1 if scheme == "center" else -(-iters // 8)  # k_hotspot_tb: 8 steps per pass
@@ -65,7 +75,9 @@ def main():
             row = {"grid": f"{side}x{side}", "iterations": iters, "scheme": scheme, "kernel": kern, "ms": ms,
                    "us_per_step": 1e3 * ms / iters, "quality_mre": q, "hbm_passes": passes,
                    "algorithmic_gbs": 12.0 * px * passes / (ms * 1e-3) / 1e9,
-                   "speedup_vs_exact": res["exact"] / ms}
+                   "speedup_vs_exact": res["exact"] / ms,
+                   "unblocked_kernel": kern1, "unblocked_us_per_step": 1e3 * ms1 / iters,
+                   "unblocked_gbs": 12.0 * px * iters / (ms1 * 1e-3) / 1e9, "blocked_speedup": ms1 / ms}
             print(json.dumps(row), flush=True)
             rows.append(row)
         del td, pd, out, exact
