@@ -119,14 +119,7 @@ static const Plan& cand_plan(paraprox_filter f, const Candidate& c) {
     return is_skip_scheme(c.scheme) ? get_plan_skip(f, c.dy, c.dx) : get_plan(f, c.dy, c.dx);
 }
 
-bool fused_quality_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("PARAPROX_FUSED_QUALITY");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+bool fused_quality_enabled() { return knobs().fused_quality; }
 
 constexpr int kMaxLatticeReach = 1 << 20;
 
@@ -477,14 +470,7 @@ paraprox_status paraprox_tune_lattice(paraprox_filter f, const float* d_train, c
     return paraprox_tune_lattice_decide(parts, m, toq, out_scheme, out_reach, out_quality);
 }
 
-static bool hotspot_tb_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("PARAPROX_HOTSPOT_TB");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+static bool hotspot_tb_enabled() { return knobs().hotspot_tb; }
 
 paraprox_status paraprox_hotspot(const paraprox_hotspot_params* prm, paraprox_scheme scheme, int reach,
                                  const float* d_temp, const float* d_power, float* d_out, const paraprox_image* img,

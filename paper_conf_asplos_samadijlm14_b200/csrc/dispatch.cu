@@ -14,10 +14,6 @@
 
 #include "k_tiles.cuh"
 
-#ifndef PPX_TILE_CHUNK_DEFAULT
-#define PPX_TILE_CHUNK_DEFAULT 16
-#endif
-
 namespace ppx {
 
 cudaError_t launch_generic(const Plan& p, const float* in, const View& v, float* out, long long opitch,
@@ -88,35 +84,14 @@ void init_registry() {
     });
 }
 
-bool force_generic() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("PARAPROX_FORCE_GENERIC");
-        v = (e && e[0] == '1') ? 1 : 0;
-    }
-    return v == 1;
-}
+bool force_generic() { return knobs().force_generic; }
 
 }  // namespace
 
-// tiles per CTA of the plain tile kernels (k_tiles.cuh, bounded persistence);
-// PARAPROX_TILE_CHUNK=0 keeps the fully persistent grid
-static int tile_chunk() {
-    static const int v = [] {
-        const char* e = std::getenv("PARAPROX_TILE_CHUNK");
-        const int c = e ? std::atoi(e) : PPX_TILE_CHUNK_DEFAULT;
-        return c > 0 ? c : INT_MAX;
-    }();
-    return v;
-}
+// tiles per CTA of the plain tile kernels (k_tiles.cuh, bounded persistence)
+static int tile_chunk() { return knobs().tile_chunk; }
 
-bool tma_store_enabled() {
-    static const bool v = [] {
-        const char* e = std::getenv("PARAPROX_TMA_STORE");
-        return !(e && e[0] == '0');
-    }();
-    return v;
-}
+bool tma_store_enabled() { return knobs().tma_store; }
 
 void register_tile_instance(const TileInstance& ti) {
     for (const Entry& o : reg())  // the same instance serves several radii
@@ -144,7 +119,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     const int box_w = kTW + 2 * round4(e.ti.hx), box_h = kTH + 2 * e.ti.hy;
     if (!encode_tmap_3d(&tmap, in + (long long)v.lo * v.pitch, v.w, rows_valid, v.n, v.pitch, fstride, box_w, box_h))
         return cudaSuccess;
-    // output map for the TMA-store epilogue (PPX_TMA_STORE); a layout it
+    // output map for the TMA-store epilogue (PARAPROX_TMA_STORE); a layout it
     // cannot describe keeps the register-store epilogue
     CUtensorMap omap = tmap;  // (unused unless A.tma_store)
     const bool tma_store = !qo && !add && tma_store_enabled() &&

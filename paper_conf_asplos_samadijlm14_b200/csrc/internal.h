@@ -134,6 +134,12 @@ cudaError_t launch_quality(const float* e, const float* a, const View& v, parapr
 constexpr int kQualityBlocks = 1184;  // partial-count cap of the persistent (tile, map) quality grids
 // scratch (doubles) launch_quality and launch_stencil_quality need for an
 // image of `count` pixels: one partial pair per CTA
+// environment settings, read once (knobs.cpp)
+struct Knobs {
+    bool force_generic = false, fused_quality = true, tma_store = true, hotspot_tb = true;
+    int tile_chunk = 16, lattice_chunk = 8;  // INT_MAX = fully persistent
+};
+const Knobs& knobs();
 size_t quality_scratch_doubles(long long count);
 // partial pairs that scratch holds (a quality grid must not exceed it)
 size_t quality_scratch_pairs(long long count);

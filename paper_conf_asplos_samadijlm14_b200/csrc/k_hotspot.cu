@@ -35,9 +35,7 @@ namespace ppx {
 
 constexpr int kHsBH = 48, kHsBW = 128, kHsWarps = 8, kHsRPW = kHsBH / kHsWarps, kHsMaxS = 8;
 constexpr int kHsThreads = 32 * kHsWarps;
-#ifndef PPX_HS_MINB
-#define PPX_HS_MINB 3  // CTAs per SM the register budget is sized for
-#endif
+constexpr int kHsMinBlocks = 3;  // CTAs per SM the register budget is sized for
 
 struct HsArgs {
     int n, h, w;
@@ -116,28 +114,46 @@ __device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[k
                 wl = __shfl_up_sync(0xffffffffu, cur.w, 1);
                 er = __shfl_down_sync(0xffffffffu, cur.x, 1);
             }
-            float4 nv;
+            // the taps in order (N, W, C, E, S), column pairs (0,1) and (2,3)
+            // in FFMA2 lanes where the operand pair is a register pair
+            // (rows above / below, the centre, P); the west / east operands
+            // straddle the pairs and take scalar FFMAs -- the same fp32 fma
+            // per cell either way
+            float2 a01 = make_float2(0.f, 0.f), a23 = make_float2(0.f, 0.f);
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                const float x = hs_get(cur, c);
-                float acc = 0.f;
-                bool first = true;
+            for (int a = -HY; a <= HY; ++a)
 #pragma unroll
-                for (int a = -HY; a <= HY; ++a)
-#pragma unroll
-                    for (int b = -HX; b <= HX; ++b) {
-                        if (a != 0 && b != 0) continue;
-                        float v;
-                        if (a < 0) v = hs_get(nrt, c);
-                        else if (a > 0) v = hs_get(sth, c);
-                        else if (b < 0) v = wst[c] ? x : (c == 0 ? wl : hs_get(cur, c - 1));
-                        else if (b > 0) v = est[c] ? x : (c == 3 ? er : hs_get(cur, c + 1));
-                        else v = x;
-                        acc = __fmaf_rn(A.w9[a + 1][b + 1], v, first ? 0.f : acc);
-                        first = false;
+                for (int b = -HX; b <= HX; ++b) {
+                    if (a != 0 && b != 0) continue;
+                    const float wt = A.w9[a + 1][b + 1];
+                    if (b == 0) {
+                        const float4 v = a < 0 ? nrt : (a > 0 ? sth : cur);
+                        const float2 w2 = make_float2(wt, wt);
+                        a01 = __ffma2_rn(w2, make_float2(v.x, v.y), a01);
+                        a23 = __ffma2_rn(w2, make_float2(v.z, v.w), a23);
+                    } else {
+                        float v0, v1, v2, v3;  // the west (b < 0) or east neighbours
+                        if (b < 0) {
+                            v0 = wst[0] ? cur.x : wl;
+                            v1 = wst[1] ? cur.y : cur.x;
+                            v2 = wst[2] ? cur.z : cur.y;
+                            v3 = wst[3] ? cur.w : cur.z;
+                        } else {
+                            v0 = est[0] ? cur.x : cur.y;
+                            v1 = est[1] ? cur.y : cur.z;
+                            v2 = est[2] ? cur.z : cur.w;
+                            v3 = est[3] ? cur.w : er;
+                        }
+                        a01.x = __fmaf_rn(wt, v0, a01.x);
+                        a01.y = __fmaf_rn(wt, v1, a01.y);
+                        a23.x = __fmaf_rn(wt, v2, a23.x);
+                        a23.y = __fmaf_rn(wt, v3, a23.y);
                     }
-                hs_set(nv, c, __fadd_rn(__fmaf_rn(A.alpha, hs_get(Pv[i], c), acc), A.beta));
-            }
+                }
+            const float2 al2 = make_float2(A.alpha, A.alpha), be2 = make_float2(A.beta, A.beta);
+            a01 = __fadd2_rn(__ffma2_rn(al2, make_float2(Pv[i].x, Pv[i].y), a01), be2);
+            a23 = __fadd2_rn(__ffma2_rn(al2, make_float2(Pv[i].z, Pv[i].w), a23), be2);
+            const float4 nv = make_float4(a01.x, a01.y, a23.x, a23.y);
             prev = cur;
             T[i] = nv;
         }
@@ -145,7 +161,7 @@ __device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[k
 }
 
 template <int HY, int HX>
-__global__ void __launch_bounds__(kHsThreads, PPX_HS_MINB) k_hotspot_tb(const __grid_constant__ HsArgs A) {
+__global__ void __launch_bounds__(kHsThreads, kHsMinBlocks) k_hotspot_tb(const __grid_constant__ HsArgs A) {
     using G = HsGeom<HY, HX>;
     extern __shared__ __align__(16) float bnd[];
     const int wi = threadIdx.x >> 5, lane = threadIdx.x & 31;

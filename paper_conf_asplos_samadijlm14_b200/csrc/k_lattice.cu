@@ -30,9 +30,7 @@
 
 #include "k_tiles.cuh"
 
-#ifndef PPX_LAT_MIN_BLOCKS
-#define PPX_LAT_MIN_BLOCKS 2
-#endif
+constexpr int kLatMinBlocks = 2;  // CTAs per SM the register budget is sized for
 
 namespace ppx {
 
@@ -42,7 +40,9 @@ constexpr int lat_m(int S, int t) { return floor_div(2 * t + S, 2 * S); }
 
 template <int S, int R>
 struct LGeom {
-    static constexpr int RB = S * ((8 + S / 2) / S > 0 ? (8 + S / 2) / S : 1);  // rows per thread
+    // rows per thread: a multiple of S near 8 (6 for S = 3: an even count for
+    // the row-pair form below within the register budget of 2 CTAs per SM)
+    static constexpr int RB = S == 3 ? 6 : S * ((8 + S / 2) / S > 0 ? (8 + S / 2) / S : 1);
     static constexpr int TH = kWarps * RB;                                     // tile rows
     static constexpr int QT = TH / S;                                          // row groups per tile
     static constexpr int QR = RB / S;                                          // row groups per thread
@@ -75,14 +75,26 @@ struct LatArgs {
     int stride, chunk;  // tile schedule, as TileArgs (bounded persistence)
 };
 
+// Row-pair form for the dense s = 3 lattice (the compute-bound one: 27-36
+// FMAs per output for a 9x9 filter on 5.33 B/px): FFMA2 lanes hold output
+// rows (y, y+1) of one column, as in k_tiles.cuh's row pairs; the staged
+// value is the broadcast operand and the weight pair comes from wp, so no
+// odd-column operand is rebuilt.  Per-output tap order (staged row, then
+// column offset) is that of the column-pair form: bit-identical.
+template <int S, bool SEP>
+__host__ __device__ constexpr bool lat_row_pairs() { return !SEP && S == 3; }
+
 struct LatW {
+    // row pairs: wp[phi][m - MLO][b + 4] = (w[phi][m][b], w[phi'][m'][b]) with
+    // (phi', m') the phase and relative accessed row of the next output row
+    float2 wp[3][4][9];
     float w[9][4][9];  // dense: [phase][m - MLO][b + 4]
     float wy[9][4];    // separable: [phase][m - MLO]
     float wx[9];       // separable: [b + 4]
 };
 
 template <int S, int R, bool SEP>
-__global__ void __launch_bounds__(kThreads, PPX_LAT_MIN_BLOCKS) k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A,
+__global__ void __launch_bounds__(kThreads, kLatMinBlocks) k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A,
                                                          const __grid_constant__ LatW W) {
     using G = LGeom<S, R>;
     constexpr int HX = R, HXP = G::HXP, SW = G::SW, AB = G::AB, RB = G::RB, TH = G::TH, MLO = G::MLO;
@@ -161,7 +173,54 @@ __global__ void __launch_bounds__(kThreads, PPX_LAT_MIN_BLOCKS) k_lattice(const 
 #pragma unroll
         for (int k = 0; k < RB; ++k) acc[k][0] = acc[k][1] = make_float2(0.f, 0.f);
 
-        if constexpr (!SEP) {
+        if constexpr (lat_row_pairs<S, SEP>()) {
+            static_assert(RB % 2 == 0, "row pairs need an even RB");
+            float2 rp[RB / 2][4];  // rp[p][c] = outputs (rows 2p, 2p+1) of column c
+#pragma unroll
+            for (int p = 0; p < RB / 2; ++p)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) rp[p][c] = make_float2(0.f, 0.f);
+            static_for<G::QR + G::NA - 1>([&](auto TT) {
+                constexpr int tt = decltype(TT)::value;
+                const int sr = min(max(tq0 + tt, rlo), rhi);
+                float v[NV];
+                const float4* p4 = reinterpret_cast<const float4*>(Sm + sr * SW) + lane;
+#pragma unroll
+                for (int q = 0; q < NV / 4; ++q) {
+                    const float4 t = p4[q];
+                    v[4 * q] = t.x, v[4 * q + 1] = t.y, v[4 * q + 2] = t.z, v[4 * q + 3] = t.w;
+                }
+                static_for<RB / 2>([&](auto KP) {
+                    constexpr int p = decltype(KP)::value, k0 = 2 * p, k1 = 2 * p + 1;
+                    constexpr int phi0 = k0 % S, m0 = tt - k0 / S + MLO;
+                    constexpr int phi1 = k1 % S, m1 = tt - k1 / S + MLO;
+                    constexpr bool u0 = m0 >= MLO && m0 <= G::MHI && lat_used<S, R>(phi0, m0);
+                    constexpr bool u1 = m1 >= MLO && m1 <= G::MHI && lat_used<S, R>(phi1, m1);
+                    if constexpr (u0 || u1) {
+                        static_for<2 * HX + 1>([&](auto B) {
+                            constexpr int b = decltype(B)::value - HX;
+#pragma unroll
+                            for (int c = 0; c < 4; ++c) {
+                                const float xv = v[HXP + b + c];
+                                if constexpr (u0 && u1)
+                                    rp[p][c] = __ffma2_rn(W.wp[phi0][m0 - MLO][b + 4], make_float2(xv, xv), rp[p][c]);
+                                else if constexpr (u0)
+                                    rp[p][c].x = __fmaf_rn(W.w[phi0][m0 - MLO][b + 4], xv, rp[p][c].x);
+                                else
+                                    rp[p][c].y = __fmaf_rn(W.w[phi1][m1 - MLO][b + 4], xv, rp[p][c].y);
+                            }
+                        });
+                    }
+                });
+            });
+#pragma unroll
+            for (int p = 0; p < RB / 2; ++p) {
+                acc[2 * p][0] = make_float2(rp[p][0].x, rp[p][1].x);
+                acc[2 * p][1] = make_float2(rp[p][2].x, rp[p][3].x);
+                acc[2 * p + 1][0] = make_float2(rp[p][0].y, rp[p][1].y);
+                acc[2 * p + 1][1] = make_float2(rp[p][2].y, rp[p][3].y);
+            }
+        } else if constexpr (!SEP) {
             static_for<G::QR + G::NA - 1>([&](auto TT) {
                 constexpr int tt = decltype(TT)::value;  // staged row tq0 + tt
                 const int sr = min(max(tq0 + tt, rlo), rhi);
@@ -314,28 +373,10 @@ static const LatInstance* find_lat(int s, int r, bool sep) {
     return nullptr;
 }
 
-// tiles per CTA (bounded persistence, k_tiles.cuh); PARAPROX_LATTICE_CHUNK=0
-// keeps the fully persistent grid
-#ifndef PPX_LAT_CHUNK_DEFAULT
-#define PPX_LAT_CHUNK_DEFAULT 8
-#endif
-static int lattice_chunk() {
-    static const int v = [] {
-        const char* e = std::getenv("PARAPROX_LATTICE_CHUNK");
-        const int c = e ? std::atoi(e) : PPX_LAT_CHUNK_DEFAULT;
-        return c > 0 ? c : INT_MAX;
-    }();
-    return v;
-}
+// tiles per CTA (bounded persistence, k_tiles.cuh)
+static int lattice_chunk() { return knobs().lattice_chunk; }
 
-static bool lattice_force_generic() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("PARAPROX_FORCE_GENERIC");
-        v = (e && e[0] == '1') ? 1 : 0;
-    }
-    return v == 1;
-}
+static bool lattice_force_generic() { return knobs().force_generic; }
 
 static cudaError_t launch_lattice_generic(const paraprox_filter_s& lf, const float* in, const View& v, float* out,
                                           long long opitch, long long ofs, int dy, int dx, cudaStream_t s) {
@@ -429,6 +470,13 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
     }
     if (lf.separable)
         for (int j = 0; j < lf.kx; ++j) W.wx[j - r + 4] = lf.wx[j];
+    if (S == 3 && !lf.separable)  // row-pair weights (lat_row_pairs)
+        for (int phi = 0; phi < S; ++phi)
+            for (int m = 0; m <= e->mhi - e->mlo; ++m) {
+                const int phi1 = (phi + 1) % S, m1 = m - (phi == S - 1 ? 1 : 0);
+                for (int b = 0; b < 9; ++b)
+                    W.wp[phi][m][b] = make_float2(W.w[phi][m][b], m1 >= 0 ? W.w[phi1][m1][b] : 0.f);
+            }
     const long long cap = (long long)nsm * occ;
     long long grid = nt < cap ? nt : cap;
     A.stride = (int)grid;

@@ -17,24 +17,11 @@
 
 namespace ppx {
 
-#ifndef PPX_PU
-#define PPX_PU 4
-#endif
-constexpr int kPU = PPX_PU;
+constexpr int kPU = 4;  // float4 loads in flight per thread
 static_assert(kPU >= 4, "quality_scratch_doubles() sizes one partial pair per 4096 floats");
 
-// streaming 128-bit load: evict-first, or with a 256-byte L2 prefetch hint
-__device__ __forceinline__ float4 ld_stream(const float4* p) {
-#if PPX_MAP_L2PF
-    float4 v;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0, %1, %2, %3}, [%4];"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-                 : "l"(p));
-    return v;
-#else
-    return __ldcs(p);
-#endif
-}
+// streaming 128-bit load, evict-first
+__device__ __forceinline__ float4 ld_stream(const float4* p) { return __ldcs(p); }
 
 template <bool SEP>
 __device__ __forceinline__ float pw(float x, float w0, float w1) {

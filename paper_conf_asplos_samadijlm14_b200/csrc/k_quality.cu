@@ -42,10 +42,7 @@ static cudaError_t launch_pdl(void (*k)(KArgs...), int grid, int block, cudaStre
 // the map kernel; tools/qbench.cu measured this 13-18 % faster at 64 MiB per
 // image than the persistent grid-stride loop it replaced (equal at 1 GiB).
 // Other layouts walk rows.
-#ifndef PPX_QU
-#define PPX_QU 4
-#endif
-constexpr int kQU = PPX_QU;
+constexpr int kQU = 4;  // float4 loads of each image in flight per thread
 constexpr long long kQChunk = 256LL * kQU * 4;  // floats of each image per CTA
 static_assert(kQU >= 4, "quality_scratch_doubles() sizes one partial pair per 4096 floats");
 

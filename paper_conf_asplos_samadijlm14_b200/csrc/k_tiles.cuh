@@ -33,24 +33,14 @@
 #include "quality.cuh"
 #include "tma.cuh"
 
-#ifndef PPX_TILE_MAX_STAGES
-#define PPX_TILE_MAX_STAGES 3
-#endif
-#ifndef PPX_TILE_MIN_BLOCKS
-#define PPX_TILE_MIN_BLOCKS 2
-#endif
+constexpr int kTileMaxStages = 3;  // TMA ring depth where shared memory allows
+constexpr int kTileMinBlocks = 2;  // CTAs per SM of most instances (tile_min_blocks)
 
 namespace ppx {
 
 constexpr int kTW = 128;                 // tile width (outputs)
-#ifndef PPX_KRB
-#define PPX_KRB 8
-#endif
-#ifndef PPX_KWARPS
-#define PPX_KWARPS 8
-#endif
-constexpr int kRB = PPX_KRB;             // output rows per thread
-constexpr int kWarps = PPX_KWARPS;       // 256 threads
+constexpr int kRB = 8;                   // output rows per thread
+constexpr int kWarps = 8;                // 256 threads
 constexpr int kTH = kRB * kWarps;        // 64 tile rows
 constexpr int kThreads = 32 * kWarps;
 
@@ -111,10 +101,10 @@ __host__ __device__ constexpr int tile_min_blocks() {
                      (HY == 3 && HX == 4 && MASKY == L3 && MASKX == F4) ||
                      (HY == 4 && HX == 4 && MASKY == L4 && MASKX == L4)))
                ? 3
-               : PPX_TILE_MIN_BLOCKS;
+               : kTileMinBlocks;
 }
 
-template <int HY, int HX, int MINB = PPX_TILE_MIN_BLOCKS>
+template <int HY, int HX, int MINB = kTileMinBlocks>
 struct Geom {
     static constexpr int HXP = round4(HX);
     static constexpr int SW = kTW + 2 * HXP;   // staged row length (floats)
@@ -125,7 +115,7 @@ struct Geom {
     // 3: 2 stages)
     static constexpr int FIT = (110 * 1024) / STAGE_STRIDE;
     static constexpr int STAGES =
-        MINB >= 3 ? 2 : (FIT < 2 ? 2 : (FIT < PPX_TILE_MAX_STAGES ? FIT : PPX_TILE_MAX_STAGES));
+        MINB >= 3 ? 2 : (FIT < 2 ? 2 : (FIT < kTileMaxStages ? FIT : kTileMaxStages));
     static constexpr int SMEM = STAGES * STAGE_STRIDE;
 };
 
@@ -164,13 +154,10 @@ __device__ __forceinline__ void load_pairs(const float* row, int lane, float2 (&
 // pairs (v[I0], v[I0+1]) straddle two 64-bit registers; ptxas builds them
 // with MOVs, which take FMA-pipe cycles of their own (ncu), so four scalar
 // FFMAs -- the same issue slots, fewer pipe cycles, same fp32 fma per lane --
-// are used instead (PPX_ODD_PAIRS=1 keeps the pair form, A/B; kbench at c4
-// and c3: lattice +4-12 %, separable exact +21 %, dense column-pair instances
-// within +-5 % except dense_l3_f4, 14 % slower, which keeps the pair form).
-#ifndef PPX_ODD_PAIRS
-#define PPX_ODD_PAIRS 0
-#endif
-template <int NV, int I0, bool ODD_PAIRS = PPX_ODD_PAIRS>
+// are used instead (r01 A/B of the pair form, kbench at c4 and c3: lattice
+// +4-12 %, separable exact +21 %, dense column-pair instances within +-5 %
+// except dense_l3_f4, 14 % slower, which keeps the pair form).
+template <int NV, int I0, bool ODD_PAIRS = false>
 __device__ __forceinline__ void fma_pairs(float2 (&acc)[2], float w, const float2 (&ve)[NV / 2],
                                           const float2 (&vo)[NV / 2 - 1]) {
     const float2 w2 = make_float2(w, w);
@@ -252,9 +239,6 @@ __host__ __device__ constexpr bool use_row_pairs() {
     bool full = HY >= 1, odd = false;
     for (int a = -HY; a <= HY; ++a) full = full && ((MASKY >> (a + 8)) & 1u);
     for (int b = -HX; b <= HX; ++b) odd = odd || (((MASKX >> (b + 8)) & 1u) && (b & 1));
-#ifdef PPX_NO_ROW_PAIRS  // A/B only
-    full = false;
-#endif
     return full && odd;
 }
 
@@ -305,8 +289,8 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     // the CTA's k-th tile: strided (b + k G: concurrently running CTAs take
-    // neighbouring tiles) or, with PPX_TILE_RUNS, a contiguous run of tiles
-    // along the rows (a tile's left halo was fetched by the same CTA just before)
+    // neighbouring tiles; r01 A/B: contiguous runs of tiles per CTA were 1.10x
+    // the DRAM reads and slower at small batches)
     //
     // Bounded persistence (A.chunk < INT_MAX): a fully persistent grid lets
     // its CTAs drift apart over hundreds of tiles, so the tiles in flight no
@@ -315,19 +299,12 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
     // chunks, each CTA takes `chunk` tiles of the stride pattern and retires;
     // the block scheduler starts the next wave's CTAs in order as slots free
     // up, which keeps the window compact.
-#if PPX_TILE_RUNS
-    const int per = (A.ntiles + gridDim.x - 1) / gridDim.x;
-    const int t_begin = blockIdx.x * per, t_end = min(A.ntiles, t_begin + per);
-    auto tile_at = [&](int k) { return t_begin + k; };
-    auto in_range = [&](int t) { return t < t_end; };
-#else
     const int wave = (int)blockIdx.x / A.stride;
     const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
     const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
                                                : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
     auto tile_at = [&](int k) { return (int)min(t_base + (long long)k * A.stride, (long long)INT_MAX); };
     auto in_range = [&](int t) { return t < t_end; };
-#endif
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s) {
             const int t = tile_at(s);
@@ -473,7 +450,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
                             static_for<2 * HX + 1>([&](auto B) {
                                 constexpr int b = decltype(B)::value - HX;
                                 if constexpr (has(MASKX, b))
-                                    fma_pairs<NV, HXP + b, PPX_ODD_PAIRS || odd_pairs_faster<HY, HX, MASKY, MASKX>()>(
+                                    fma_pairs<NV, HXP + b, odd_pairs_faster<HY, HX, MASKY, MASKX>()>(
                                         acc[k], W.w[a + 4][b + 4], ve, vo);
                             });
                         }
@@ -539,11 +516,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
                 for (int c = 0; c < 4; ++c)
                     if (x + c < A.w) racc.add(A.metric, A.ref_exact ? q4[c] : r4[c], A.ref_exact ? r4[c] : q4[c]);
             }
-#ifdef PPX_NO_SPECIAL_EPI  // A/B only: the plain store epilogue
-        } else if (false) {
-#else
         } else if (A.addp) {
-#endif
             float r[kRB][4];
 #pragma unroll
             for (int k = 0; k < kRB; ++k) {

@@ -22,19 +22,9 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
     return fn;
 }
 
-// L2 promotion of the TMA loads; PARAPROX_TMA_L2PROMO = 0 / 64 / 128 / 256
-// overrides it (A/B only)
-static CUtensorMapL2promotion l2_promotion() {
-    static CUtensorMapL2promotion v = [] {
-        const char* e = std::getenv("PARAPROX_TMA_L2PROMO");
-        const int b = e ? std::atoi(e) : 256;
-        return b == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
-               : b == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
-               : b == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
-                          : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
-    }();
-    return v;
-}
+// L2 promotion of the TMA loads: 256 B (r01 A/B of none / 64 / 128 / 256 B:
+// within +-1 %)
+static CUtensorMapL2promotion l2_promotion() { return CU_TENSOR_MAP_L2_PROMOTION_L2_256B; }
 
 bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n, long long pitch,
                     long long fstride, int box_w, int box_h) {

@@ -15,10 +15,13 @@ final CTA.  Three comparisons per workload:
    0.95, 0.99 identical (train on the first 10 runs and
    keep the first kernel meeting the TOQ; L572-592);
 2. the same fused partials vs `oracle.quality` on the GPU's own stored fp32
-   outputs (exact and candidate) within 1e-12: isolates the reduction, whose
-   only difference from the oracle is fp64 summation order;
+   outputs (exact and candidate) within RTOL_REDUCTION: isolates the
+   reduction, whose only difference from the oracle is the fp64 summation
+   order (a tree on the GPU, rows in sequence in the oracle: typically
+   sqrt(N) 2^-53 ~ 1e-12 relative at N = 8.3e7 - 1.7e8 terms; measured
+   1.26e-12 on c3's L2), so RTOL_REDUCTION = 1e-11;
 3. `paraprox_quality` (the unfused a4 kernel) vs `oracle.quality` on the same
-   stored outputs within 1e-12.
+   stored outputs within RTOL_REDUCTION.
 
 QTOL: the two sides do not compute the same fp32 outputs.  The GPU applies
 the plan's folded weights w' = fp32(sum of the substituted taps), each
@@ -38,7 +41,7 @@ from workloads import filters as F
 pytestmark = pytest.mark.gpu
 
 QTOL = 1e-8
-RTOL_REDUCTION = 1e-12
+RTOL_REDUCTION = 1e-11
 TOQS = (0.80, 0.90, 0.95, 0.99)
 
 # name: (frames, h, w, filter, metric) -- bench.py WORKLOADS / tuner training set
