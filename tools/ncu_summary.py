@@ -35,7 +35,7 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e
               "msecond": 1e-3, "ns": 1e-9, "us": 1e-6, "ms": 1e-3}
 
 
-SETS = {256: "s0", 896: "f1", 1984: "f2", 4064: "f3", 8176: "f4", 1344: "l2", 2336: "l3", 4368: "l4"}
+SETS = {256: "s0", 896: "f1", 1984: "f2", 4064: "f3", 8176: "f4", 1344: "l2", 2336: "l3", 4368: "l4", 131071: "f8"}
 
 
 def short(name):
