@@ -116,7 +116,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     const int rows_valid = v.hi - v.lo + 1;
     const long long fstride = v.n > 1 ? v.fstride : (long long)rows_valid * v.pitch;
     CUtensorMap tmap;
-    const int box_w = kTW + 2 * round4(e.ti.hx), box_h = kTH + 2 * e.ti.hy;
+    const int box_w = kTW + 2 * round4(e.ti.hx), box_h = e.ti.th + 2 * e.ti.hy;
     if (!encode_tmap_3d(&tmap, in + (long long)v.lo * v.pitch, v.w, rows_valid, v.n, v.pitch, fstride, box_w, box_h))
         return cudaSuccess;
     // output map for the TMA-store epilogue (PARAPROX_TMA_STORE); a layout it
@@ -124,7 +124,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     CUtensorMap omap = tmap;  // (unused unless A.tma_store)
     const bool tma_store = !qo && !add && tma_store_enabled() &&
                            encode_tmap_3d(&omap, out, v.w, v.h, v.n, opitch, v.n > 1 ? ofs : (long long)v.h * opitch,
-                                          kTW, kTH);
+                                          kTW, e.ti.th);
     {
         std::lock_guard<std::mutex> lk(g_mu);
         if (!e.ready[dev]) {
@@ -132,7 +132,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
             for (TileKernel fn : {e.ti.fn, e.ti.fnq}) {
                 err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, e.ti.smem);
                 if (err != cudaSuccess) return err;
-                err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(fn == e.ti.fn ? &occ : &occq, fn, kThreads,
+                err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(fn == e.ti.fn ? &occ : &occq, fn, e.ti.threads,
                                                                     e.ti.smem);
                 if (err != cudaSuccess) return err;
             }
@@ -152,7 +152,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     A.rows_valid = rows_valid;
     A.row_off = -v.lo;
     A.tiles_x = (v.w + kTW - 1) / kTW;
-    A.tiles_y = (v.h + kTH - 1) / kTH;
+    A.tiles_y = (v.h + e.ti.th - 1) / e.ti.th;
     const long long nt = (long long)A.tiles_x * A.tiles_y * v.n;
     if (nt >= (1LL << 31)) return cudaSuccess;
     A.ntiles = (int)nt;
@@ -214,7 +214,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     if (qo) qo->grid = grid;  // one partial pair per CTA, grid <= qo->cap_pairs
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(kThreads);
+    cfg.blockDim = dim3(e.ti.threads);
     cfg.dynamicSmemBytes = e.ti.smem;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];

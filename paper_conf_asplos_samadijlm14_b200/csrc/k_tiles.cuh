@@ -40,7 +40,7 @@ namespace ppx {
 
 constexpr int kTW = 128;                 // tile width (outputs)
 constexpr int kRB = 8;                   // output rows per thread
-constexpr int kWarps = 8;                // 256 threads
+constexpr int kWarps = 8;                // 256 threads (lattice kernels; tile instances: tile_warps)
 constexpr int kTH = kRB * kWarps;        // 64 tile rows
 constexpr int kThreads = 32 * kWarps;
 
@@ -93,31 +93,57 @@ __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
 // stages for the instances where the A/B measured that faster (kbench, two
 // runs: exact 5x5 +5 %, c4 rows {-3,0,3} x all columns +8 %, c4 rows/columns
 // {-4,0,4} +5 %; most other instances lose 3-7 % and the exact 9x9 15 %)
+// Warps per CTA of an instance: 8 (64-row tiles) or 4 (32-row tiles, twice
+// the CTAs per SM).  r02 kbench A/B of 4 against 8 warps on every instance
+// (profiles/r02_ab_w4.md): +1..+5 % on c1-c3 (exact 5x5 +4.8 %, separable 7x7
+// +2.5 %, c4 rows {-4,0,4} x all columns +9 %), -2..-5 % where the columns
+// are a lattice of 3 or 4 (c4 {-3,0,3}, {-4,0,4}) and -1 % on the 9x9 exact;
+// the separable radius-8 (ConvSep) instances were not measured and stay at 8.
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+__host__ __device__ constexpr int tile_warps() {
+    constexpr uint32_t F4 = 0x1FFu << 4;
+    constexpr uint32_t L3 = (1u << 5) | (1u << 8) | (1u << 11), L4 = (1u << 4) | (1u << 8) | (1u << 12);
+    if (SEP) return (HY > 4 || HX > 4) ? 8 : 4;
+    if (MASKX == L3 || MASKX == L4) return 8;
+    if (MASKY == F4 && MASKX == F4) return 8;
+    return 4;
+}
+
+// CTAs per SM an instance is built for (8-warp CTAs; twice that with 4): 2
+// (up to 3 stages), or 3 with 2 stages for the instances where the r01 A/B
+// measured that faster (kbench, two runs: exact 5x5 +5 %, c4 rows {-3,0,3} x
+// all columns +8 %, c4 rows/columns {-4,0,4} +5 %; most other instances lose
+// 3-7 % and the exact 9x9 15 %)
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
 __host__ __device__ constexpr int tile_min_blocks() {
     constexpr uint32_t F2 = 0x1Fu << 6, F4 = 0x1FFu << 4;
     constexpr uint32_t L3 = (1u << 5) | (1u << 8) | (1u << 11), L4 = (1u << 4) | (1u << 8) | (1u << 12);
-    return (!SEP && ((HY == 2 && HX == 2 && MASKY == F2 && MASKX == F2) ||
-                     (HY == 3 && HX == 4 && MASKY == L3 && MASKX == F4) ||
-                     (HY == 4 && HX == 4 && MASKY == L4 && MASKX == L4)))
-               ? 3
-               : kTileMinBlocks;
+    const int b = (!SEP && ((HY == 2 && HX == 2 && MASKY == F2 && MASKX == F2) ||
+                            (HY == 3 && HX == 4 && MASKY == L3 && MASKX == F4) ||
+                            (HY == 4 && HX == 4 && MASKY == L4 && MASKX == L4)))
+                      ? 3
+                      : kTileMinBlocks;
+    return b * (8 / tile_warps<HY, HX, MASKY, MASKX, SEP>());
 }
 
-template <int HY, int HX, int MINB = kTileMinBlocks>
+template <int HY, int HX, int MINB = kTileMinBlocks, int WARPS = 8>
 struct Geom {
+    static constexpr int TH = kRB * WARPS;     // tile rows
     static constexpr int HXP = round4(HX);
     static constexpr int SW = kTW + 2 * HXP;   // staged row length (floats)
-    static constexpr int SH = kTH + 2 * HY;    // staged rows
+    static constexpr int SH = TH + 2 * HY;     // staged rows
     static constexpr int STAGE_BYTES = SW * SH * 4;
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
-    // as many stages as fit MINB CTAs per SM (2: <= 110 KiB each, 2..MAX;
-    // 3: 2 stages)
-    static constexpr int FIT = (110 * 1024) / STAGE_STRIDE;
+    // as many stages as fit MINB CTAs per SM in ~220 KiB, 2..MAX (MINB a
+    // multiple of 3: the occupancy-3 instances, 2 stages)
+    static constexpr int FIT = (220 * 1024 / MINB) / STAGE_STRIDE;
     static constexpr int STAGES =
-        MINB >= 3 ? 2 : (FIT < 2 ? 2 : (FIT < kTileMaxStages ? FIT : kTileMaxStages));
+        MINB % 3 == 0 ? 2 : (FIT < 2 ? 2 : (FIT < kTileMaxStages ? FIT : kTileMaxStages));
     static constexpr int SMEM = STAGES * STAGE_STRIDE;
 };
+
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+using GeomOf = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>(), tile_warps<HY, HX, MASKY, MASKX, SEP>()>;
 
 __device__ __forceinline__ constexpr bool has(uint32_t mask, int off) { return (mask >> (off + 8)) & 1u; }
 
@@ -250,11 +276,13 @@ __host__ __device__ constexpr bool odd_pairs_faster() {
 }
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
-__global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASKX, SEP>())) k_tiles(const __grid_constant__ CUtensorMap tmap,
-                                                       const TileArgs A, const __grid_constant__ TapW W,
-                                                       const __grid_constant__ CUtensorMap omap) {
-    using G = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()>;
+__global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
+                                  (tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()))
+    k_tiles(const __grid_constant__ CUtensorMap tmap, const TileArgs A, const __grid_constant__ TapW W,
+            const __grid_constant__ CUtensorMap omap) {
+    using G = GeomOf<HY, HX, MASKY, MASKX, SEP>;
     constexpr int HXP = G::HXP, SW = G::SW, SH = G::SH, NV = 4 + 2 * HXP;
+    constexpr int WARPS = tile_warps<HY, HX, MASKY, MASKX, SEP>(), NT = 32 * WARPS, TH = G::TH;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ uint64_t bars[G::STAGES];
 
@@ -265,7 +293,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
         f = t / tiles_per_frame;
         const int r = t - f * tiles_per_frame;
         const int ty = r / A.tiles_x;
-        y0 = ty * kTH;
+        y0 = ty * TH;
         x0 = (r - ty * A.tiles_x) * kTW;
     };
     auto issue = [&](int t, int s) {
@@ -356,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
         if (HY > 0 && (drow0 < 0 && A.ntop > 0 || drow0 + SH > A.rows_valid && A.nbot > 0)) {
             // stripe-edge tile: the halo rows come from the peer pointers
             // (TMA zero-filled them), columns clamped to the image
-            for (int idx = tid; idx < SH * SW; idx += kThreads) {
+            for (int idx = tid; idx < SH * SW; idx += NT) {
                 const int r = idx / SW, c = idx - r * SW;
                 const int dr = drow0 + r;
                 const float* src = nullptr;
@@ -372,7 +400,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
         if (clo > 0 || chi < SW - 1) {  // border columns: replicate the edge (clamp)
             // only the out-of-image columns are touched: at most HXP per side
             const int nl = clo, nr = SW - 1 - chi, nb = nl + nr;
-            for (int idx = tid; idx < SH * nb; idx += kThreads) {
+            for (int idx = tid; idx < SH * nb; idx += NT) {
                 const int r = idx / nb, c = idx - r * nb;
                 if (c < nl) S[r * SW + c] = S[r * SW + clo];
                 else S[r * SW + chi + 1 + (c - nl)] = S[r * SW + chi];
@@ -459,11 +487,11 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
             });
         } else {
             // horizontal pass over the staged rows (clamped), kept in registers
-            constexpr int RPT = (SH + kWarps - 1) / kWarps;  // rows per thread
+            constexpr int RPT = (SH + WARPS - 1) / WARPS;  // rows per thread
             float2 hz[RPT][2];
 #pragma unroll
             for (int q = 0; q < RPT; ++q) {
-                const int r = wi + q * kWarps;
+                const int r = wi + q * WARPS;
                 if (r < SH) {
                     const int sr = min(max(r, rlo), rhi);
                     float2 ve[NV / 2], vo[NV / 2 - 1];
@@ -478,7 +506,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
             __syncthreads();  // every thread has read its rows: overwrite in place
 #pragma unroll
             for (int q = 0; q < RPT; ++q) {
-                const int r = wi + q * kWarps;
+                const int r = wi + q * WARPS;
                 if (r < SH)
                     reinterpret_cast<float4*>(S + r * SW + HXP)[lane] =
                         make_float4(hz[q][0].x, hz[q][0].y, hz[q][1].x, hz[q][1].y);
@@ -528,7 +556,7 @@ __global__ void __launch_bounds__(kThreads, (tile_min_blocks<HY, HX, MASKY, MASK
             tile_epilogue_add(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0,
                               x, r);
         } else if (A.tma_store) {
-            // the tile's outputs replace its consumed input stage ([kTH][kTW])
+            // the tile's outputs replace its consumed input stage ([TH][kTW])
             // and leave as one TMA store (out-of-image elements are clipped)
             __syncthreads();  // every thread has finished reading the stage
 #pragma unroll
@@ -584,6 +612,7 @@ struct TileInstance {
     TileKernel fn;   // plain / additive-input stencil
     TileKernel fnq;  // fused-quality instance
     int smem;
+    int threads, th;  // CTA size and tile rows (tile_warps)
     const char* name;
 };
 
@@ -599,7 +628,9 @@ TileInstance make_instance(const char* name) {
     ti.hx = HX;
     ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP, false>;
     ti.fnq = k_tiles<HY, HX, MASKY, MASKX, SEP, true>;
-    ti.smem = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()>::SMEM;
+    ti.smem = GeomOf<HY, HX, MASKY, MASKX, SEP>::SMEM;
+    ti.threads = 32 * tile_warps<HY, HX, MASKY, MASKX, SEP>();
+    ti.th = GeomOf<HY, HX, MASKY, MASKX, SEP>::TH;
     ti.name = name;
     return ti;
 }
