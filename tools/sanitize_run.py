@@ -51,6 +51,11 @@ def main():
     for scheme, reach in (("exact", 0), ("row", 1), ("col", 1), ("center", 1)):
         P.hotspot(td, pd, H.PARAMS, scheme, reach, 1)
         P.hotspot(td, pd, H.PARAMS, scheme, reach, 11)
+    # a grid with interior tiles of the temporally blocked kernel (no clamp)
+    t2, p2 = H.frames(1, 200, 300, 3)
+    t2d, p2d = torch.from_numpy(t2).cuda(), torch.from_numpy(p2).cuda()
+    for scheme, reach in (("exact", 0), ("row", 1), ("col", 1)):
+        P.hotspot(t2d, p2d, H.PARAMS, scheme, reach, 8)
     rt = P.Runtime(P.Filter(F.mean(5)), 0.9, "mre", check_every=2)
     rt.train(x)
     out = torch.empty_like(x)
