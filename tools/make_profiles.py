@@ -96,8 +96,20 @@ def main():
         md = os.path.join(OUT, f"ncu_full_{wl}.md")
         if os.path.exists(md):
             shutil.copy(md, os.path.join(PROF, f"{tag}_ncu_full_{wl}.md"))
-    if os.path.exists(os.path.join(OUT, "launches_c2.md")):
-        shutil.copy(os.path.join(OUT, "launches_c2.md"), os.path.join(PROF, f"{tag}_launches_c2.md"))
+    for wl in ("c2", "c3"):
+        if os.path.exists(os.path.join(OUT, f"launches_{wl}.md")):
+            shutil.copy(os.path.join(OUT, f"launches_{wl}.md"), os.path.join(PROF, f"{tag}_launches_{wl}.md"))
+    for name in ("ncu_kernels_c3.md", "ncu_bytes.md", "bench_ref.json"):
+        if os.path.exists(os.path.join(OUT, name)):
+            shutil.copy(os.path.join(OUT, name), os.path.join(PROF, f"{tag}_{name}"))
+    sani = [os.path.join(OUT, f"sanitize_{t}.log") for t in ("memcheck", "racecheck", "synccheck", "initcheck")]
+    if all(os.path.exists(x) for x in sani):
+        lines = [f"# compute-sanitizer over tools/sanitize_run.py — {tag}", ""]
+        for x in sani:
+            txt = open(x).read().splitlines()
+            keep = [ln for ln in txt if "SUMMARY" in ln or "sanitize run ok" in ln]
+            lines.append(f"* `{os.path.basename(x)[9:-4]}`: " + "; ".join(keep))
+        open(os.path.join(PROF, f"{tag}_sanitizers.md"), "w").write("\n".join(lines) + "\n")
     box = os.path.join(OUT, "traffic_box.json")
     if os.path.exists(box):
         tj = os.path.join(PROF, "traffic.json")

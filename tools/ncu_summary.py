@@ -73,7 +73,7 @@ def launches(path):
         order.append((k, v))
     tot = sum(t for _, t in agg.values())
     print(f"# ncu launch list: {os.path.basename(path)}\n")
-    print("`ncu --metrics gpu__time_duration.sum --clock-control none -c 400` (cold-cache, serialised:"
+    print("`ncu --metrics gpu__time_duration.sum --clock-control none` over the bench command (cold-cache, serialised:"
           " compare shares, not absolutes).\n")
     print(f"{len(order)} launches, {tot * 1e3:.3f} ms total\n")
     print("| kernel | launches | total us | mean us | share |")
