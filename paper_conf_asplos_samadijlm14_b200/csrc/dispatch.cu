@@ -116,7 +116,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     const int rows_valid = v.hi - v.lo + 1;
     const long long fstride = v.n > 1 ? v.fstride : (long long)rows_valid * v.pitch;
     CUtensorMap tmap;
-    const int box_w = kTW + 2 * round4(e.ti.hx), box_h = e.ti.th + 2 * e.ti.hy;
+    const int box_w = e.ti.sw, box_h = e.ti.th + 2 * e.ti.hy;
     if (!encode_tmap_3d(&tmap, in + (long long)v.lo * v.pitch, v.w, rows_valid, v.n, v.pitch, fstride, box_w, box_h))
         return cudaSuccess;
     // output map for the TMA-store epilogue (PARAPROX_TMA_STORE); a layout it
@@ -182,6 +182,10 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     if (p.separable) {
         for (int i = 0; i < p.ny; ++i) W.wy[p.ay[i] + 8] = p.wyf[i];
         for (int j = 0; j < p.nx; ++j) W.wx[p.ax[j] + 8] = p.wxf[j];
+        for (int b = 1; b < 17; ++b) {  // weight pairs of the wide separable path
+            W.wxp[b] = make_float2(W.wx[b], W.wx[b - 1]);
+            W.wyp[b] = make_float2(W.wy[b], W.wy[b - 1]);
+        }
     } else {
         for (int i = 0; i < p.ny; ++i)
             for (int j = 0; j < p.nx; ++j) W.w[p.ay[i] + 4][p.ax[j] + 4] = p.wf[i * p.nx + j];

@@ -52,6 +52,8 @@ struct TapW {
     float w[9][9];   // dense folded weights at [a + 4][b + 4]   (r <= 4)
     float wy[17];    // separable folded weights at [a + 8]     (r <= 8)
     float wx[17];
+    // wide separable path (sep_wide): weight pairs (w[b], w[b - 1]) at [b + 8]
+    float2 wyp[17], wxp[17];
 };
 
 struct TileArgs {
@@ -126,11 +128,19 @@ __host__ __device__ constexpr int tile_min_blocks() {
     return b * (8 / tile_warps<HY, HX, MASKY, MASKX, SEP>());
 }
 
-template <int HY, int HX, int MINB = kTileMinBlocks, int WARPS = 8>
+// Separable filters wider than 9 taps (the paper's ConvSep 1x17 loops): the
+// horizontal pass with one staged row per lane (below), on a row pitch padded
+// to 4 mod 8 words so that the 8 lanes of a 128-bit access hit distinct banks.
+template <int HX, bool SEP>
+__host__ __device__ constexpr bool sep_wide() { return SEP && HX > 4; }
+
+template <int HY, int HX, int MINB = kTileMinBlocks, int WARPS = 8, bool PAD = false>
 struct Geom {
-    static constexpr int TH = kRB * WARPS;     // tile rows
+    // tile rows (the wide separable path: 48, so that its 64 staged rows are
+    // two full warp-rows of the horizontal pass)
+    static constexpr int TH = PAD ? 48 : kRB * WARPS;
     static constexpr int HXP = round4(HX);
-    static constexpr int SW = kTW + 2 * HXP;   // staged row length (floats)
+    static constexpr int SW = kTW + 2 * HXP + (PAD ? 4 : 0);  // staged row length (floats)
     static constexpr int SH = TH + 2 * HY;     // staged rows
     static constexpr int STAGE_BYTES = SW * SH * 4;
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) & ~127;
@@ -143,7 +153,8 @@ struct Geom {
 };
 
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
-using GeomOf = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>(), tile_warps<HY, HX, MASKY, MASKX, SEP>()>;
+using GeomOf = Geom<HY, HX, tile_min_blocks<HY, HX, MASKY, MASKX, SEP>(), tile_warps<HY, HX, MASKY, MASKX, SEP>(),
+                    sep_wide<HX, SEP>()>;
 
 __device__ __forceinline__ constexpr bool has(uint32_t mask, int off) { return (mask >> (off + 8)) & 1u; }
 
@@ -355,8 +366,20 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
         coords(tile, f, y0, x0);
         const int ty0 = wi * kRB;
         const int x = x0 + 4 * lane;
-        float4 qv[Q ? kRB : 1];  // Q: this thread's reference values, in flight during the FMAs
-        if constexpr (Q) {
+        constexpr bool WIDE = sep_wide<HX, SEP>();
+        constexpr int WR = TH / 2;   // wide path: output rows per thread (column tid % 128)
+        const int wc = tid & (kTW - 1), wh = tid >> 7;
+        float qw[Q && WIDE ? WR : 1];  // wide Q: reference values of the thread's column
+        if constexpr (Q && WIDE) {
+            const float* rb = A.refp + (long long)f * A.rfs + x0 + wc;
+#pragma unroll
+            for (int k = 0; k < WR; ++k) {
+                const int y = y0 + WR * wh + k;
+                qw[k] = (y < A.h && x0 + wc < A.w) ? __ldcs(rb + (long long)y * A.rpitch) : 0.f;
+            }
+        }
+        float4 qv[Q && !WIDE ? kRB : 1];  // Q: this thread's reference values, in flight during the FMAs
+        if constexpr (Q && !WIDE) {
             const float* rb = A.refp + (long long)f * A.rfs + x;
 #pragma unroll
             for (int k = 0; k < kRB; ++k) {
@@ -485,6 +508,108 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
                     });
                 }
             });
+        } else if constexpr (WIDE) {
+            // Wide separable filters (ConvSep's 1x17 loops; r01: 0.63 of the
+            // copy peak, bound by shared-memory bandwidth: a lane's 4 outputs
+            // read a 20-float window, ~55 B of LDS/STS traffic per output).
+            // Horizontal pass: warp w takes output columns [16w, 16w + 16),
+            // lane l the staged rows l and l + 32: a 32-float window per 16
+            // outputs (row pitch padded to 4 mod 8 words: the 8 lanes of a
+            // 128-bit access hit distinct banks), each staged column feeding
+            // output pairs (j, j + 1) through one FFMA2 with the weight pair
+            // (wx[b], wx[b - 1]).  Vertical pass: thread t takes column
+            // t % 128 and 24 consecutive output rows, each staged row feeding
+            // row pairs (k, k + 1) likewise; outputs leave from registers.
+            // Rows outside the valid staged rows are not computed: the
+            // vertical pass clamps its row index instead (their horizontal
+            // result equals the edge row's).  Per output the taps run in the
+            // plain path's order (columns, then rows, ascending): the same
+            // fp32 fma sequence, bit-identical.
+            static_assert(WARPS == 8 && SH <= 64, "sep_wide: 8 warps x 16 columns, <= 2 x 32 staged rows");
+            constexpr int NW = 16 + 2 * HXP;  // window floats per 16 outputs
+            const int cw = 16 * wi;
+#pragma unroll
+            for (int q = 0; q < (SH + 31) / 32; ++q) {
+                const int r = lane + 32 * q;
+                const bool live = r < SH && r >= rlo && r <= rhi;
+                float2 h2[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) h2[j] = make_float2(0.f, 0.f);
+                if (live) {
+                    float v[NW];
+                    const float4* p4 = reinterpret_cast<const float4*>(S + r * SW + cw);
+#pragma unroll
+                    for (int k = 0; k < NW / 4; ++k) {
+                        const float4 t = p4[k];
+                        v[4 * k] = t.x, v[4 * k + 1] = t.y, v[4 * k + 2] = t.z, v[4 * k + 3] = t.w;
+                    }
+                    static_for<NW>([&](auto T) {
+                        constexpr int t = decltype(T)::value;
+                        static_for<8>([&](auto J) {
+                            constexpr int j = 2 * decltype(J)::value;
+                            constexpr int b0 = t - HXP - j, b1 = b0 - 1;
+                            constexpr bool u0 = b0 >= -HX && b0 <= HX && has(MASKX, b0);
+                            constexpr bool u1 = b1 >= -HX && b1 <= HX && has(MASKX, b1);
+                            if constexpr (u0 && u1)
+                                h2[j / 2] = __ffma2_rn(W.wxp[b0 + 8], make_float2(v[t], v[t]), h2[j / 2]);
+                            else if constexpr (u0)
+                                h2[j / 2].x = __fmaf_rn(W.wx[b0 + 8], v[t], h2[j / 2].x);
+                            else if constexpr (u1)
+                                h2[j / 2].y = __fmaf_rn(W.wx[b1 + 8], v[t], h2[j / 2].y);
+                        });
+                    });
+                }
+                __syncthreads();  // every warp has read rows lane + 32 q: write them back in place
+                if (live) {
+                    float4* o4 = reinterpret_cast<float4*>(S + r * SW + HXP + cw);
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                        o4[k] = make_float4(h2[2 * k].x, h2[2 * k].y, h2[2 * k + 1].x, h2[2 * k + 1].y);
+                }
+            }
+            __syncthreads();
+            // vertical pass: column wc, output rows [WR wh, WR wh + WR)
+            float2 vp[WR / 2];
+#pragma unroll
+            for (int k = 0; k < WR / 2; ++k) vp[k] = make_float2(0.f, 0.f);
+            auto vpass = [&](auto clamped) {
+                static_for<WR + 2 * HY>([&](auto M) {
+                    constexpr int m = decltype(M)::value;  // staged row WR wh + m
+                    const int sr = decltype(clamped)::value ? min(max(WR * wh + m, rlo), rhi) : WR * wh + m;
+                    const float hv = S[sr * SW + HXP + wc];
+                    static_for<WR / 2>([&](auto KP) {
+                        constexpr int k = 2 * decltype(KP)::value;
+                        constexpr int a0 = m - HY - k, a1 = a0 - 1;
+                        constexpr bool u0 = a0 >= -HY && a0 <= HY && has(MASKY, a0);
+                        constexpr bool u1 = a1 >= -HY && a1 <= HY && has(MASKY, a1);
+                        if constexpr (u0 && u1)
+                            vp[k / 2] = __ffma2_rn(W.wyp[a0 + 8], make_float2(hv, hv), vp[k / 2]);
+                        else if constexpr (u0)
+                            vp[k / 2].x = __fmaf_rn(W.wy[a0 + 8], hv, vp[k / 2].x);
+                        else if constexpr (u1)
+                            vp[k / 2].y = __fmaf_rn(W.wy[a1 + 8], hv, vp[k / 2].y);
+                    });
+                });
+            };
+            if (rlo == 0 && rhi == SH - 1) vpass(std::false_type{});
+            else vpass(std::true_type{});
+            const int xo = x0 + wc;
+            if constexpr (Q) {
+#pragma unroll
+                for (int k = 0; k < WR; ++k) {
+                    const float rv = (k & 1) ? vp[k / 2].y : vp[k / 2].x;
+                    if (y0 + WR * wh + k < A.h && xo < A.w)
+                        racc.add(A.metric, A.ref_exact ? qw[k] : rv, A.ref_exact ? rv : qw[k]);
+                }
+            } else if (xo < A.w) {
+                float* ob = A.out + (long long)f * A.ofs + (long long)(y0 + WR * wh) * A.opitch + xo;
+                const int nrow = min(WR, A.h - (y0 + WR * wh));
+#pragma unroll
+                for (int k = 0; k < WR; ++k) {
+                    if (k < nrow) __stcs(ob, (k & 1) ? vp[k / 2].y : vp[k / 2].x);
+                    ob += A.opitch;
+                }
+            }
         } else {
             // horizontal pass over the staged rows (clamped), kept in registers
             constexpr int RPT = (SH + WARPS - 1) / WARPS;  // rows per thread
@@ -533,7 +658,9 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
         // stores: a TMA tensor store per tile or 128-bit streaming stores; the
         // additive-input epilogue lives out of line so the plain stencils keep
         // a lean epilogue (and their register budget)
-        if constexpr (Q) {
+        if constexpr (WIDE) {
+            // stored / compared in the wide separable branch
+        } else if constexpr (Q) {
 #pragma unroll
             for (int k = 0; k < kRB; ++k) {
                 const int y = y0 + ty0 + k;
@@ -613,6 +740,7 @@ struct TileInstance {
     TileKernel fnq;  // fused-quality instance
     int smem;
     int threads, th;  // CTA size and tile rows (tile_warps)
+    int sw;           // staged row length = the TMA box width (floats)
     const char* name;
 };
 
@@ -631,6 +759,7 @@ TileInstance make_instance(const char* name) {
     ti.smem = GeomOf<HY, HX, MASKY, MASKX, SEP>::SMEM;
     ti.threads = 32 * tile_warps<HY, HX, MASKY, MASKX, SEP>();
     ti.th = GeomOf<HY, HX, MASKY, MASKX, SEP>::TH;
+    ti.sw = GeomOf<HY, HX, MASKY, MASKX, SEP>::SW;
     ti.name = name;
     return ti;
 }

@@ -78,7 +78,7 @@ def test_dense_all_reaches(P, O, name, w, shape):
         assert_dense(P, O, x, w, dy, dx, f)
 
 
-@pytest.mark.parametrize("ky,kx", [(7, 7), (3, 5), (1, 17), (17, 1), (9, 9)])
+@pytest.mark.parametrize("ky,kx", [(7, 7), (3, 5), (1, 17), (17, 1), (9, 9), (17, 17), (5, 11)])
 @pytest.mark.parametrize("shape", [(2, 77, 300), (1, 190, 700)], ids=["2x77x300", "1x190x700"])
 def test_separable_all_reaches(P, O, ky, kx, shape):
     wy = F.conv(1, seed=40 + ky, ky=ky).ravel()
