@@ -159,7 +159,7 @@ def oracle_host_threads():
     return n
 
 
-def cpu_baseline(wl, kind, w, scheme, reach, budget_s=10.0, max_reps=400):
+def cpu_baseline(wl, kind, w, scheme, reach, budget_s=10.0, max_reps=5000):
     """The oracle as it stands, on the host cores, over a bounded sample of the
     workload: whole frames (or a row band of the c4 image) until ~budget_s."""
     import oracle
