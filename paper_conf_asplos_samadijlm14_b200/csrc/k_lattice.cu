@@ -38,12 +38,18 @@ constexpr int floor_div(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) /
 // nearest accessed row of window row phi + i, relative: floor((phi+i)/s + 1/2)
 constexpr int lat_m(int S, int t) { return floor_div(2 * t + S, 2 * S); }
 
-template <int S, int R>
+// Warps per CTA: 4 for the dense lattices, 8 for the separable ones (r02
+// kbench A/B of 4 against 8 warps: dense +1..+12 % except s = 3 / 7 at c4
+// (-1..-2 %); separable -0.3..-1 %, profiles/r02_ab_w4.md)
+template <bool SEP>
+__host__ __device__ constexpr int lat_warps() { return SEP ? 8 : 4; }
+
+template <int S, int R, int WARPS = kWarps>
 struct LGeom {
     // rows per thread: a multiple of S near 8 (6 for S = 3: an even count for
     // the row-pair form below within the register budget of 2 CTAs per SM)
     static constexpr int RB = S == 3 ? 6 : S * ((8 + S / 2) / S > 0 ? (8 + S / 2) / S : 1);
-    static constexpr int TH = kWarps * RB;                                     // tile rows
+    static constexpr int TH = WARPS * RB;                                      // tile rows
     static constexpr int QT = TH / S;                                          // row groups per tile
     static constexpr int QR = RB / S;                                          // row groups per thread
     static constexpr int MLO = lat_m(S, -R);
@@ -94,9 +100,10 @@ struct LatW {
 };
 
 template <int S, int R, bool SEP>
-__global__ void __launch_bounds__(kThreads, kLatMinBlocks) k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A,
-                                                         const __grid_constant__ LatW W) {
-    using G = LGeom<S, R>;
+__global__ void __launch_bounds__(32 * lat_warps<SEP>(), kLatMinBlocks * 8 / lat_warps<SEP>())
+    k_lattice(const __grid_constant__ CUtensorMap tmap, const LatArgs A, const __grid_constant__ LatW W) {
+    constexpr int WARPS = lat_warps<SEP>(), NT = 32 * WARPS;
+    using G = LGeom<S, R, WARPS>;
     constexpr int HX = R, HXP = G::HXP, SW = G::SW, AB = G::AB, RB = G::RB, TH = G::TH, MLO = G::MLO;
     constexpr int NV = 4 + 2 * HXP;
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -160,7 +167,7 @@ __global__ void __launch_bounds__(kThreads, kLatMinBlocks) k_lattice(const __gri
         if (clo > 0 || chi < SW - 1) {  // border columns: replicate the edge (clamp)
             // only the out-of-image columns are touched: at most HXP per side
             const int nl = clo, nr = SW - 1 - chi, nb = nl + nr;
-            for (int idx = tid; idx < AB * nb; idx += kThreads) {
+            for (int idx = tid; idx < AB * nb; idx += NT) {
                 const int r = idx / nb, c = idx - r * nb;
                 if (c < nl) Sm[r * SW + c] = Sm[r * SW + clo];
                 else Sm[r * SW + chi + 1 + (c - nl)] = Sm[r * SW + chi];
@@ -238,11 +245,11 @@ __global__ void __launch_bounds__(kThreads, kLatMinBlocks) k_lattice(const __gri
                 });
             });
         } else {
-            constexpr int RPT = (AB + kWarps - 1) / kWarps;
+            constexpr int RPT = (AB + WARPS - 1) / WARPS;
             float2 hz[RPT][2];
 #pragma unroll
             for (int q = 0; q < RPT; ++q) {
-                const int r = wi + q * kWarps;
+                const int r = wi + q * WARPS;
                 if (r < AB) {
                     const int sr = min(max(r, rlo), rhi);
                     float2 ve[NV / 2], vo[NV / 2 - 1];
@@ -257,7 +264,7 @@ __global__ void __launch_bounds__(kThreads, kLatMinBlocks) k_lattice(const __gri
             __syncthreads();
 #pragma unroll
             for (int q = 0; q < RPT; ++q) {
-                const int r = wi + q * kWarps;
+                const int r = wi + q * WARPS;
                 if (r < AB)
                     reinterpret_cast<float4*>(Sm + r * SW + HXP)[lane] =
                         make_float4(hz[q][0].x, hz[q][0].y, hz[q][1].x, hz[q][1].y);
@@ -348,13 +355,15 @@ struct LatInstance {
     bool sep;
     LatKernel fn;
     int smem, ab, th, mlo, mhi;
+    int threads;
     const char* name;
 };
 
 template <int S, int R, bool SEP>
 LatInstance make_lat(const char* name) {
-    using G = LGeom<S, R>;
-    return LatInstance{S, R, SEP, k_lattice<S, R, SEP>, G::SMEM, G::AB, G::TH, G::MLO, G::MHI, name};
+    using G = LGeom<S, R, lat_warps<SEP>()>;
+    return LatInstance{S, R, SEP, k_lattice<S, R, SEP>, G::SMEM, G::AB, G::TH, G::MLO, G::MHI,
+                       32 * lat_warps<SEP>(), name};
 }
 
 static const LatInstance* find_lat(int s, int r, bool sep) {
@@ -425,7 +434,7 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
         if (!occ) {
             err = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, e->smem);
             if (err != cudaSuccess) return err;
-            err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, e->fn, kThreads, e->smem);
+            err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, e->fn, e->threads, e->smem);
             if (err != cudaSuccess) return err;
             if (occ < 1) occ = 1;
             if (dev < 64 && idx >= 0 && idx < 32) occ_cache[dev][idx] = occ;
@@ -488,7 +497,7 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
-    cfg.blockDim = dim3(kThreads);
+    cfg.blockDim = dim3(e->threads);
     cfg.dynamicSmemBytes = e->smem;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];

@@ -428,3 +428,36 @@ def test_fused_quality_many_tiny_frames(P, O):
     for k, (s, r) in enumerate(cands):
         an = P.stencil_approx(xd, f, s, r).cpu().numpy()
         assert abs(qg[k] - O.quality(en, an, "mre")) <= 1e-12, (s, r)
+
+
+def test_wide_separable_layouts_and_stripes(P, O):
+    """The wide separable path (17-tap loops, `sep_wide`): aligned pitched and
+    strided layouts (pitch 532 > w, frame stride > h * pitch) against the
+    oracle, and row stripes with halo rows bitwise equal to the whole image
+    (the stripe-edge tiles clamp at their valid rows)."""
+    wy = F.conv(1, seed=61, ky=17).ravel()
+    wx = F.conv(17, seed=62, ky=1).ravel()
+    f = P.Filter(wy=wy, wx=wx)
+    x = W.frames(3, 150, 520, 8)
+    big = torch.zeros((3, 170, 532), device="cuda")
+    big[:, 4:154, 8:528] = dev(x)
+    view = big[:, 4:154, 8:528]  # 16-byte aligned: the tile (TMA) path
+    outb = torch.zeros_like(big)
+    out = outb[:, 4:154, 8:528]
+    for dy, dx in [(0, 0), (3, 3), (0, 8), (8, 0), (2, 5)]:
+        g = P.stencil_approx_xy(view, f, dy, dx, out=out).cpu().numpy()
+        assert P.last_kernel().startswith("sep8_") or (dy, dx) == (2, 5), P.last_kernel()
+        o = O.stencil_sep(x, wy, wx, dy, dx)
+        bound = RTOL * O.stencil_sep(np.abs(x), np.abs(wy), np.abs(wx), dy, dx) + 1e-30
+        assert np.all(np.abs(g - o) <= bound), (dy, dx, P.last_kernel())
+        assert torch.count_nonzero(outb[:, :4]) == 0 and torch.count_nonzero(outb[:, :, :8]) == 0  # no stray writes
+    img = dev(W.image(700, 600, 9))
+    for dy, dx in [(0, 0), (3, 3)]:
+        full = P.stencil_approx_xy(img, f, dy, dx)
+        hy = f.plan_info(dy, dx)["halo_y"]
+        bounds = [0, 130, 333, 700]
+        for k in range(3):
+            r0, r1 = bounds[k], bounds[k + 1]
+            ht, hb = min(hy, r0), min(hy, 700 - r1)
+            got = P.stencil_approx_xy(img[r0 - ht:r1 + hb].clone(), f, dy, dx, halo_top=ht, halo_bottom=hb)
+            assert torch.equal(got, full[r0:r1]), (dy, dx, k)
