@@ -4,21 +4,25 @@
 // grid is partitioned into tiles that are advanced independently.  One CTA
 // advances a tile by S <= 8 time steps from a single HBM read of T and P.
 //
-// Layout: a 48 x 128 box of cells (the tile plus an 8-cell halo on the
-// accessed axes: 32 x 112 outputs for the exact stencil, 48 x 128 for the
-// row scheme, which reads no neighbour row) is held in REGISTERS: warp w owns
-// box rows 6w..6w+5, lane l columns 4l..4l+3 (T and P, 48 floats per
-// thread).  A step needs only
+// Layout: a 48 x 128 or 96 x 128 box of cells (the tile plus an 8-cell halo on
+// the accessed axes: 32 x 112 or 80 x 112 outputs for the exact stencil,
+// 48 x 128 for the row scheme, which reads no neighbour row) is held in
+// REGISTERS: warp w owns box rows 6w..6w+5 (12w..12w+11 in the tall box), lane l
+// columns 4l..4l+3 of T; P (constant over the steps) in registers too, or in
+// thread-private shared-memory slots in the tall box.  A step needs only
 //  * the west / east neighbours: the adjacent lanes' edge columns (shuffles),
-//  * the rows directly above / below a warp's six rows: the neighbouring
-//    warps publish their first and last rows in a ping-pong shared buffer
-//    (16 KB), one barrier per step.
+//  * the rows directly above / below a warp's rows: the neighbouring warps
+//    publish their first and last rows in a ping-pong shared buffer (16 KB),
+//    one barrier per step.
 // The box edge has no neighbours: those cells turn to garbage one cell per
 // step, which never reaches the outputs (8 halo cells >= S steps).  Clamp to
 // the image edge (reading S7) is applied at read time in border tiles only:
 // a cell on the first / last valid row or column reads itself in place of
 // the missing neighbour, so out-of-image cells are never read by in-image
-// ones and need no fix-up between steps.
+// ones and need no fix-up between steps.  The tall box (2 CTAs per SM instead
+// of 3) computes 1.37 cells per output instead of 1.71: it is taken for steps
+// with a row halo when it still gives every SM two tiles (8192^2 exact 47.1 ->
+// 38.9 us per step; the paper's 1024^2 keeps the 48-row box).
 //
 // Each step adds the taps in the order of the tile kernels (rows ascending,
 // columns ascending, fmaf from 0), then fmaf(alpha, P, .) + beta: bit-
@@ -33,9 +37,13 @@
 
 namespace ppx {
 
-constexpr int kHsBH = 48, kHsBW = 128, kHsWarps = 8, kHsRPW = kHsBH / kHsWarps, kHsMaxS = 8;
+constexpr int kHsBW = 128, kHsWarps = 8, kHsMaxS = 8;
 constexpr int kHsThreads = 32 * kHsWarps;
-constexpr int kHsMinBlocks = 3;  // CTAs per SM the register budget is sized for
+// box rows: 48 (6 per warp) or 96 (12 per warp: less halo overhead, 2 CTAs per
+// SM instead of 3; the launch takes it when there are at least two tiles per SM
+// and the step has a row halo)
+template <int BH>
+__host__ __device__ constexpr int hs_min_blocks() { return BH >= 96 ? 2 : 3; }
 
 struct HsArgs {
     int n, h, w;
@@ -56,11 +64,17 @@ struct HsArgs {
     long long ppitch;
 };
 
-template <int HY, int HX>
+template <int HY, int HX, int BH>
 struct HsGeom {
-    static constexpr int OH = kHsBH - 2 * kHsMaxS * HY;  // output rows per tile
+    static constexpr int RPW = BH / kHsWarps;           // box rows per warp
+    static constexpr int OH = BH - 2 * kHsMaxS * HY;     // output rows per tile
     static constexpr int OW = kHsBW - 2 * kHsMaxS * HX;  // output columns per tile
-    static constexpr int SMEM = HY ? 2 * kHsWarps * 2 * kHsBW * (int)sizeof(float) : 0;
+    // P in registers (48-row box) or, for the 96-row box, in thread-private
+    // shared slots ([row][thread] float4: conflict-free); then the ping-pong
+    // of the warps' boundary rows
+    static constexpr bool PREG = BH < 96;
+    static constexpr int PBYTES = PREG ? 0 : RPW * kHsThreads * (int)sizeof(float4);
+    static constexpr int SMEM = PBYTES + (HY ? 2 * kHsWarps * 2 * kHsBW * (int)sizeof(float) : 0);
 };
 
 __device__ __forceinline__ float hs_get(const float4& v, int c) {
@@ -75,15 +89,15 @@ __device__ __forceinline__ void hs_set(float4& v, int c, float x) {
 
 // the S steps on the registers; EDGE: the box touches a valid-row or image-
 // column edge (clamped neighbour reads), else the plain interior form
-template <int HY, int HX, bool EDGE>
-__device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[kHsRPW], const HsArgs& A,
+template <int HY, int HX, int RPW, bool EDGE, class PG>
+__device__ __forceinline__ void hs_run(float4 (&T)[RPW], PG pget, const HsArgs& A,
                                        float* bnd, int wi, int lane, int oy, int ox, int lo, int hi) {
     const int S = A.steps;
     // per-row / per-column edge flags (EDGE only)
-    bool top[kHsRPW], bot[kHsRPW], wst[4], est[4];
+    bool top[RPW], bot[RPW], wst[4], est[4];
 #pragma unroll
-    for (int i = 0; i < kHsRPW; ++i) {
-        const int gy = oy + wi * kHsRPW + i;
+    for (int i = 0; i < RPW; ++i) {
+        const int gy = oy + wi * RPW + i;
         top[i] = EDGE && gy == lo;
         bot[i] = EDGE && gy == hi;
     }
@@ -94,21 +108,21 @@ __device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[k
         est[c] = EDGE && gx == A.w - 1;
     }
     for (int k = 0; k < S; ++k) {
-        float4 up = T[0], dn = T[kHsRPW - 1];
+        float4 up = T[0], dn = T[RPW - 1];
         if constexpr (HY > 0) {
             float4* B = reinterpret_cast<float4*>(bnd + (k & 1) * (kHsWarps * 2 * kHsBW));
             B[(2 * wi) * (kHsBW / 4) + lane] = T[0];
-            B[(2 * wi + 1) * (kHsBW / 4) + lane] = T[kHsRPW - 1];
+            B[(2 * wi + 1) * (kHsBW / 4) + lane] = T[RPW - 1];
             __syncthreads();
             if (wi > 0) up = B[(2 * wi - 1) * (kHsBW / 4) + lane];
             if (wi < kHsWarps - 1) dn = B[(2 * wi + 2) * (kHsBW / 4) + lane];
         }
         float4 prev = up;  // old value of the row above
 #pragma unroll
-        for (int i = 0; i < kHsRPW; ++i) {
+        for (int i = 0; i < RPW; ++i) {
             const float4 cur = T[i];
             const float4 nrt = (HY && top[i]) ? cur : prev;
-            const float4 sth = (HY && bot[i]) ? cur : (i + 1 < kHsRPW ? T[i + 1] : dn);
+            const float4 sth = (HY && bot[i]) ? cur : (i + 1 < RPW ? T[i + 1] : dn);
             float wl = 0.f, er = 0.f;
             if constexpr (HX > 0) {
                 wl = __shfl_up_sync(0xffffffffu, cur.w, 1);
@@ -151,8 +165,9 @@ __device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[k
                     }
                 }
             const float2 al2 = make_float2(A.alpha, A.alpha), be2 = make_float2(A.beta, A.beta);
-            a01 = __fadd2_rn(__ffma2_rn(al2, make_float2(Pv[i].x, Pv[i].y), a01), be2);
-            a23 = __fadd2_rn(__ffma2_rn(al2, make_float2(Pv[i].z, Pv[i].w), a23), be2);
+            const float4 pv = pget(i);
+            a01 = __fadd2_rn(__ffma2_rn(al2, make_float2(pv.x, pv.y), a01), be2);
+            a23 = __fadd2_rn(__ffma2_rn(al2, make_float2(pv.z, pv.w), a23), be2);
             const float4 nv = make_float4(a01.x, a01.y, a23.x, a23.y);
             prev = cur;
             T[i] = nv;
@@ -160,10 +175,13 @@ __device__ __forceinline__ void hs_run(float4 (&T)[kHsRPW], const float4 (&Pv)[k
     }
 }
 
-template <int HY, int HX>
-__global__ void __launch_bounds__(kHsThreads, kHsMinBlocks) k_hotspot_tb(const __grid_constant__ HsArgs A) {
-    using G = HsGeom<HY, HX>;
-    extern __shared__ __align__(16) float bnd[];
+template <int HY, int HX, int BH>
+__global__ void __launch_bounds__(kHsThreads, hs_min_blocks<BH>()) k_hotspot_tb(const __grid_constant__ HsArgs A) {
+    using G = HsGeom<HY, HX, BH>;
+    constexpr int kHsRPW = G::RPW;
+    extern __shared__ __align__(16) float smem_hs[];
+    float4* Ps = reinterpret_cast<float4*>(smem_hs) + threadIdx.x;  // this thread's P slots, stride kHsThreads
+    float* bnd = smem_hs + G::PBYTES / (int)sizeof(float);
     const int wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
     int t = blockIdx.x;
     const int f = t / (A.tiles_x * A.tiles_y);
@@ -174,17 +192,22 @@ __global__ void __launch_bounds__(kHsThreads, kHsMinBlocks) k_hotspot_tb(const _
     const float* Tf = A.t + (long long)f * A.fs;
     const float* Pf = A.p + (long long)f * A.fs;
 
-    // stage: every load of the thread's 6 x 4 cells of T and P in flight at
-    // once; cells outside the valid rows / image columns read as 0 (never
-    // used by an in-image cell)
-    float4 T[kHsRPW], Pv[kHsRPW];
+    // stage: the thread's 12 x 4 cells of T into registers (all loads in
+    // flight at once) and of P into its shared slots (cp.async, no
+    // registers); cells outside the valid rows / image columns read as 0
+    // (never used by an in-image cell)
+    float4 T[kHsRPW], Pv[G::PREG ? kHsRPW : 1];
     const int gx = ox + 4 * lane;
     const bool vec_ok = A.vec && gx >= 0 && gx + 3 < A.w;
 #pragma unroll
     for (int i = 0; i < kHsRPW; ++i) {
         const int gy = oy + wi * kHsRPW + i;
-        T[i] = Pv[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (gy < lo || gy > hi) continue;
+        T[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if constexpr (G::PREG) Pv[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (gy < lo || gy > hi) {
+            if constexpr (!G::PREG) Ps[i * kHsThreads] = make_float4(0.f, 0.f, 0.f, 0.f);
+            continue;
+        }
         const float *ts, *ps;
         if (gy < 0) {
             const long long g = (long long)(A.ntop + gy) * A.ppitch;
@@ -201,20 +224,34 @@ __global__ void __launch_bounds__(kHsThreads, kHsMinBlocks) k_hotspot_tb(const _
         }
         if (vec_ok) {
             T[i] = __ldcs(reinterpret_cast<const float4*>(ts + gx));
-            Pv[i] = __ldg(reinterpret_cast<const float4*>(ps + gx));
+            if constexpr (G::PREG) {
+                Pv[i] = __ldg(reinterpret_cast<const float4*>(ps + gx));
+            } else {
+                const uint32_t pdst = (uint32_t)__cvta_generic_to_shared(Ps + i * kHsThreads);
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(pdst), "l"(ps + gx) : "memory");
+            }
         } else {
+            float4 pv = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
             for (int c = 0; c < 4; ++c)
                 if (gx + c >= 0 && gx + c < A.w) {
                     hs_set(T[i], c, ts[gx + c]);
-                    hs_set(Pv[i], c, ps[gx + c]);
+                    hs_set(pv, c, ps[gx + c]);
                 }
+            if constexpr (G::PREG) Pv[i] = pv;
+            else Ps[i * kHsThreads] = pv;
         }
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    asm volatile("cp.async.wait_group 0;" ::: "memory");  // own slots only: no barrier needed
 
-    const bool edge = oy <= lo || oy + kHsBH - 1 >= hi || ox <= 0 || ox + kHsBW - 1 >= A.w - 1;
-    if (edge) hs_run<HY, HX, true>(T, Pv, A, bnd, wi, lane, oy, ox, lo, hi);
-    else hs_run<HY, HX, false>(T, Pv, A, bnd, wi, lane, oy, ox, lo, hi);
+    const bool edge = oy <= lo || oy + BH - 1 >= hi || ox <= 0 || ox + kHsBW - 1 >= A.w - 1;
+    auto pget = [&](int i) -> float4 {
+        if constexpr (G::PREG) return Pv[i];
+        else return Ps[i * kHsThreads];
+    };
+    if (edge) hs_run<HY, HX, kHsRPW, true>(T, pget, A, bnd, wi, lane, oy, ox, lo, hi);
+    else hs_run<HY, HX, kHsRPW, false>(T, pget, A, bnd, wi, lane, oy, ox, lo, hi);
 
     // the tile's outputs: box rows [8 HY, 8 HY + OH), columns [8 HX, 8 HX + OW)
     float* Of = A.out + (long long)f * A.fs;
@@ -275,7 +312,17 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
     A.vec = al(t) && al(pw) && al(out) && (v.pitch & 3) == 0 && (v.n == 1 || (fs & 3) == 0) &&
             (!peer || ((peer->pitch & 3) == 0 && al(peer->top_t) && al(peer->top_p) && al(peer->bot_t) &&
                        al(peer->bot_p)));
-    const int oh = p.hy ? HsGeom<1, 0>::OH : HsGeom<0, 0>::OH, ow = p.hx ? HsGeom<0, 1>::OW : HsGeom<0, 0>::OW;
+    static int nsm = 0;
+    if (!nsm) {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) !=
+                                                      cudaSuccess)
+            nsm = 148;
+    }
+    auto tiles = [&](int oh, int ow) { return (long long)((v.h + oh - 1) / oh) * ((v.w + ow - 1) / ow) * v.n; };
+    const int ow = p.hx ? HsGeom<0, 1, 48>::OW : HsGeom<0, 0, 48>::OW;
+    const bool tall = p.hy && tiles(HsGeom<1, 0, 96>::OH, ow) >= 2LL * nsm;
+    const int oh = !p.hy ? HsGeom<0, 0, 48>::OH : tall ? HsGeom<1, 0, 96>::OH : HsGeom<1, 0, 48>::OH;
     A.tiles_x = (v.w + ow - 1) / ow;
     A.tiles_y = (v.h + oh - 1) / oh;
     const long long nt = (long long)A.tiles_x * A.tiles_y * v.n;
@@ -287,10 +334,12 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
         return cudaGetLastError();
     };
     cudaError_t e;
-    if (p.hy && p.hx) e = launch(k_hotspot_tb<1, 1>, HsGeom<1, 1>::SMEM);
-    else if (p.hy) e = launch(k_hotspot_tb<1, 0>, HsGeom<1, 0>::SMEM);
-    else if (p.hx) e = launch(k_hotspot_tb<0, 1>, HsGeom<0, 1>::SMEM);
-    else e = launch(k_hotspot_tb<0, 0>, HsGeom<0, 0>::SMEM);
+    if (p.hy && p.hx) e = tall ? launch(k_hotspot_tb<1, 1, 96>, HsGeom<1, 1, 96>::SMEM)
+                               : launch(k_hotspot_tb<1, 1, 48>, HsGeom<1, 1, 48>::SMEM);
+    else if (p.hy) e = tall ? launch(k_hotspot_tb<1, 0, 96>, HsGeom<1, 0, 96>::SMEM)
+                            : launch(k_hotspot_tb<1, 0, 48>, HsGeom<1, 0, 48>::SMEM);
+    else if (p.hx) e = launch(k_hotspot_tb<0, 1, 48>, HsGeom<0, 1, 48>::SMEM);
+    else e = launch(k_hotspot_tb<0, 0, 48>, HsGeom<0, 0, 48>::SMEM);
     if (e != cudaSuccess) return e;
     count_launch(p.hy && p.hx ? "hotspot_tb_f1_f1" : p.hy ? "hotspot_tb_f1_s0" : p.hx ? "hotspot_tb_s0_f1"
                                                                                         : "hotspot_tb_s0_s0");

@@ -105,8 +105,8 @@ def test_fused_centre_steps_equal_single_steps(P):
 
 
 @pytest.mark.parametrize("scheme", ["exact", "row", "col"])
-@pytest.mark.parametrize("shape", [(2, 96, 160), (1, 20, 50), (1, 300, 700), (1, 33, 129)],
-                         ids=["2x96x160", "1x20x50", "1x300x700", "1x33x129"])
+@pytest.mark.parametrize("shape", [(2, 96, 160), (1, 20, 50), (1, 300, 700), (1, 33, 129), (2, 2050, 2047)],
+                         ids=["2x96x160", "1x20x50", "1x300x700", "1x33x129", "2x2050x2047_tall_box"])
 def test_temporal_blocking_equals_single_steps(P, scheme, shape):
     """k_hotspot_tb advances up to 8 steps per pass from one read; with the
     clamp re-applied after every step it is bit-identical to single steps."""

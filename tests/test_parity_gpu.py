@@ -461,3 +461,45 @@ def test_wide_separable_layouts_and_stripes(P, O):
             ht, hb = min(hy, r0), min(hy, 700 - r1)
             got = P.stencil_approx_xy(img[r0 - ht:r1 + hb].clone(), f, dy, dx, halo_top=ht, halo_bottom=hb)
             assert torch.equal(got, full[r0:r1]), (dy, dx, k)
+
+
+def test_concurrent_streams_and_threads(P):
+    """The library keeps no global mutable state on the data path (scratch is
+    stream-ordered, plans are cached behind a lock): four host threads, each
+    on its own stream, run stencils, qualities and the tuner concurrently on
+    different filters and frames; every result equals the sequential one."""
+    import threading
+
+    jobs = [(F.mean(5), "mre", 0), (F.conv(9), "l2", 1), (F.gaussian(3), "mre", 2), (F.separable(7), "l2", 3)]
+    frames = [dev(W.frames(3, 512, 640, 10 * k)) for k in range(4)]
+    torch.cuda.synchronize()
+
+    def work(k, res):
+        w, m, _ = jobs[k]
+        f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            x = frames[k]
+            out = []
+            for _ in range(3):
+                e = P.stencil_exact(x, f, stream=s)
+                a = P.stencil_approx(x, f, "center", 1, stream=s)
+                q = P.quality(e, a, m, stream=s)
+                t = P.tune(x, f, 0.9, m, stream=s)
+                s.synchronize()
+                out.append((e.cpu(), a.cpu(), q, t))
+            res[k] = out
+
+    seq = {}
+    for k in range(4):
+        work(k, seq)
+    par = {}
+    ths = [threading.Thread(target=work, args=(k, par)) for k in range(4)]
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join()
+    for k in range(4):
+        for (e0, a0, q0, t0), (e1, a1, q1, t1) in zip(seq[k], par[k]):
+            assert torch.equal(e0, e1) and torch.equal(a0, a1), k
+            assert q0 == q1 and t0 == t1, (k, q0, q1, t0, t1)
