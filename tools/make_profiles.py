@@ -61,16 +61,19 @@ def hotspot_md(rows, tag):
     out = [f"# NEXT-4: HotSpot (Table 1 L1648: 1024², Stencil-Partition, MRE) — {tag}", "",
            "`python tools/hotspot.py` on one B200: `iterations` steps in one `paraprox_hotspot` call, captured in a "
            "CUDA graph and replayed (CUDA events). Exact, row and column schemes run the temporally blocked kernel "
-           "(`hotspot_tb_*`: 8 steps per HBM pass, bit-identical to single steps); the centre scheme at full reach "
-           "reads no neighbour and fuses all steps into one pass (`dense_map`). quality = 1 − MRE of the final "
+           "(`hotspot_tb_*`: up to 8 steps per HBM pass, bit-identical to single steps); the centre scheme at full "
+           "reach reads no neighbour and fuses all steps into one pass (`dense_map`). quality = 1 − MRE of the final "
            "temperature against the exact iteration. `alg. GB/s` = 12 B/px × HBM passes / time (the blocked kernels "
-           "are SMEM/issue-bound, not HBM-bound).", "",
-           "| grid | steps | scheme | kernel | µs / step | quality | HBM passes | alg. GB/s | speedup |",
-           "|---|---:|---|---|---:|---:|---:|---:|---:|"]
+           "are FMA/issue-bound, not HBM-bound). *unblocked* = one `paraprox_hotspot` call (one tile-kernel pass) per "
+           "step, the same scheme; *blocked ×* = unblocked ÷ blocked time.", "",
+           "| grid | steps | scheme | kernel | µs / step | quality | HBM passes | alg. GB/s | speedup vs exact | "
+           "unblocked kernel | unblocked µs / step | blocked × |",
+           "|---|---:|---|---|---:|---:|---:|---:|---:|---|---:|---:|"]
     for r in rows:
-        out.append("| %s | %d | %s | `%s` | %.2f | %.5f | %d | %.0f | %.2f |" % (
+        out.append("| %s | %d | %s | `%s` | %.2f | %.5f | %d | %.0f | %.2f | `%s` | %.1f | %.2f |" % (
             r["grid"], r["iterations"], r["scheme"], r["kernel"], r["us_per_step"], r["quality_mre"], r["hbm_passes"],
-            r["algorithmic_gbs"], r["speedup_vs_exact"]))
+            r["algorithmic_gbs"], r["speedup_vs_exact"], r.get("unblocked_kernel", "-"),
+            r.get("unblocked_us_per_step", float("nan")), r.get("blocked_speedup", float("nan"))))
     return "\n".join(out) + "\n"
 
 
