@@ -224,26 +224,38 @@ __device__ __forceinline__ void static_for(F&& f) {
 }
 
 // Out-of-line epilogue of the additive input (HotSpot's power: out = acc +
-// alpha * p + beta), kept out of the plain stencils' register budget.
+// alpha * p + beta), kept out of the plain stencils' register budget.  All
+// kRB rows of p are requested before the first is used (one dependent round
+// trip per tile instead of one per row).
 static __device__ __noinline__ void tile_epilogue_add(const float* addp, long long apitch, long long afs, float alpha,
                                                       float beta, float* out, long long opitch, long long ofs, int h,
                                                       int w, int f, int yb, int x, const float (&r)[kRB][4]) {
+    float4 a4[kRB];
+    const bool full = x + 3 < w;
+#pragma unroll
+    for (int k = 0; k < kRB; ++k) {
+        const int y = yb + k;
+        a4[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (y >= h || x >= w) continue;
+        const float* ap = addp + (long long)f * afs + x + (long long)y * apitch;
+        if (full) {
+            a4[k] = __ldcs(reinterpret_cast<const float4*>(ap));
+        } else {
+            a4[k].x = ap[0];
+            if (x + 1 < w) a4[k].y = ap[1];
+            if (x + 2 < w) a4[k].z = ap[2];
+        }
+    }
+#pragma unroll
     for (int k = 0; k < kRB; ++k) {
         const int y = yb + k;
         if (y >= h || x >= w) continue;
-        float r4[4] = {r[k][0], r[k][1], r[k][2], r[k][3]};
-        const float* ap = addp + (long long)f * afs + x + (long long)y * apitch;
-        float a4[4] = {0.f, 0.f, 0.f, 0.f};
-        if (x + 3 < w) {
-            const float4 t = __ldcs(reinterpret_cast<const float4*>(ap));
-            a4[0] = t.x, a4[1] = t.y, a4[2] = t.z, a4[3] = t.w;
-        } else {
-            for (int c = 0; c < 4; ++c)
-                if (x + c < w) a4[c] = ap[c];
-        }
-        for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(alpha, a4[c], r4[c]), beta);
+        const float av[4] = {a4[k].x, a4[k].y, a4[k].z, a4[k].w};
+        float r4[4];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) r4[c] = __fadd_rn(__fmaf_rn(alpha, av[c], r[k][c]), beta);
         float* o = out + (long long)f * ofs + (long long)y * opitch + x;
-        if (x + 3 < w) {
+        if (full) {
             __stcs(reinterpret_cast<float4*>(o), make_float4(r4[0], r4[1], r4[2], r4[3]));
         } else {
             for (int c = 0; c < 4; ++c)
