@@ -200,6 +200,7 @@ TUNE_CASES = [
     ("mean5", F.mean(5), "mre", (10, 256, 256)),
     ("conv9", F.conv(9), "l2", (10, 256, 256)),
     ("sep7", F.separable(7), "l2", (10, 216, 384)),
+    ("sep17", F.separable(17, 3, 4), "l2", (6, 200, 300)),  # the wide separable path (ConvSep loops)
 ]
 
 
@@ -307,7 +308,8 @@ import workloads as W
 from workloads import filters as F
 P = pkg.paraprox
 out = {}
-for name, w, m in [("mean5", F.mean(5), "mre"), ("conv9", F.conv(9), "l2"), ("sep7", F.separable(7), "l2")]:
+for name, w, m in [("mean5", F.mean(5), "mre"), ("conv9", F.conv(9), "l2"), ("sep7", F.separable(7), "l2"),
+                   ("sep17", F.separable(17, 3, 4), "l2")]:
     f = P.Filter(wy=w[0], wx=w[1]) if isinstance(w, tuple) else P.Filter(w)
     x = torch.from_numpy(W.frames(4, 160, 200, 3)).cuda()
     out[name] = P.tune_partials(x, f, m).tolist()
@@ -322,7 +324,7 @@ print(json.dumps(out))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
         assert r.returncode == 0, r.stderr
         res[flag] = json.loads(r.stdout.strip().splitlines()[-1])
-    metric = {"mean5": "mre", "conv9": "l2", "sep7": "l2"}
+    metric = {"mean5": "mre", "conv9": "l2", "sep7": "l2", "sep17": "l2"}
     for name in res["1"]:
         a, b = np.array(res["1"][name]), np.array(res["0"][name])
         mt = metric[name.split("_")[0]]
