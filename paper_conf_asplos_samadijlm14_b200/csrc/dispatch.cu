@@ -89,7 +89,12 @@ bool force_generic() { return knobs().force_generic; }
 }  // namespace
 
 // tiles per CTA of the plain tile kernels (k_tiles.cuh, bounded persistence)
-static int tile_chunk() { return knobs().tile_chunk; }
+// (r02 kbench sweep of 1, 2, 3, 4, 6, 16: 4-warp instances +3..+11 % at 4
+// against 16 on c1-c4; 8-warp instances -2..-9 % below 16)
+static int tile_chunk(int threads) {
+    const int k = knobs().tile_chunk;
+    return k ? k : (threads <= 128 ? 4 : 16);
+}
 
 bool tma_store_enabled() { return knobs().tma_store; }
 
@@ -202,7 +207,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     // persistent.  A wave of `grid` CTAs takes grid * chunk tiles.
     const int taps = p.separable ? p.ny + p.nx : p.ny * p.nx;
     A.stride = grid;
-    A.chunk = taps > 45 ? INT_MAX : tile_chunk();
+    A.chunk = taps > 45 ? INT_MAX : tile_chunk(e.ti.threads);
     if (A.chunk != INT_MAX) {
         const long long waves = (nt + (long long)grid * A.chunk - 1) / ((long long)grid * A.chunk);
         if (waves * grid >= (1LL << 31)) return cudaSuccess;

@@ -137,7 +137,7 @@ constexpr int kQualityBlocks = 1184;  // partial-count cap of the persistent (ti
 // environment settings, read once (knobs.cpp)
 struct Knobs {
     bool force_generic = false, fused_quality = true, tma_store = true, hotspot_tb = true;
-    int tile_chunk = 16, lattice_chunk = 8;  // INT_MAX = fully persistent
+    int tile_chunk = 0, lattice_chunk = 4;  // INT_MAX = fully persistent; tile 0 = per instance
 };
 const Knobs& knobs();
 size_t quality_scratch_doubles(long long count);
