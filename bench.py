@@ -804,6 +804,9 @@ def main():
             "config": {
                 "workload": args.workload, "desc": wl["desc"], "frames_per_step": n, "h": h, "w": wd,
                 "filter": wl["filter"], "toq": args.toq, "metric_quality": wl["metric"],
+                "input": {"field": "1/f^beta Gaussian random field + N(0, sigma) noise, rint, clip [16, 235]",
+                          "beta": W.images.BETA, "sigma": W.images.SIGMA,
+                          "fig5_target": W.images.TARGET_FIG5},
                 "l2_defeat": f"rotating {nbuf} input/output buffer pairs ({nbuf * 8 * px_step / 2**20:.0f} MiB "
                              f"> 3x L2) so consecutive steps never hit in L2",
                 "parallelism": (f"frames x{ws}: {n} of {wl['n']} frames per rank (strong, no data-path collective)"
