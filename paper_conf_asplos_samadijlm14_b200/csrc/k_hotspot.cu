@@ -312,13 +312,10 @@ cudaError_t launch_hotspot_tb(const Plan& p, const float* t, const float* pw, fl
     A.vec = al(t) && al(pw) && al(out) && (v.pitch & 3) == 0 && (v.n == 1 || (fs & 3) == 0) &&
             (!peer || ((peer->pitch & 3) == 0 && al(peer->top_t) && al(peer->top_p) && al(peer->bot_t) &&
                        al(peer->bot_p)));
-    static int nsm = 0;
-    if (!nsm) {
-        int dev = 0;
-        if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) !=
-                                                      cudaSuccess)
-            nsm = 148;
-    }
+    int dev = 0, nsm = 0;  // the current device's SM count (a cheap attribute query)
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) !=
+                                                  cudaSuccess || nsm < 1)
+        nsm = 148;
     auto tiles = [&](int oh, int ow) { return (long long)((v.h + oh - 1) / oh) * ((v.w + ow - 1) / ow) * v.n; };
     const int ow = p.hx ? HsGeom<0, 1, 48>::OW : HsGeom<0, 0, 48>::OW;
     const bool tall = p.hy && tiles(HsGeom<1, 0, 96>::OH, ow) >= 2LL * nsm;
