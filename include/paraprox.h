@@ -170,8 +170,10 @@ PARAPROX_API paraprox_status paraprox_stencil_skip_xy(paraprox_filter f, int ski
  * h-1 from d_bot (pitch src_pitch elements) -- device pointers that may map a
  * neighbouring GPU's stripe over NVLink (paraprox_ipc_open), read inside the
  * stencil kernel with no separate collective.  0 rows = the image edge
- * (clamp).  Only the plan's halo h_y rows are read.  The caller orders the
- * neighbours' writes before this call (e.g. a barrier).  Asynchronous on s. */
+ * (clamp).  Only the plan's halo h_y rows are read; a neighbour with
+ * 0 < rows < h_y is INVALID_ARG (its first row is not the image edge, so no
+ * clamp would be correct).  The caller orders the neighbours' writes before
+ * this call (e.g. a barrier).  Asynchronous on s. */
 PARAPROX_API paraprox_status paraprox_stencil_peer(paraprox_filter f, paraprox_scheme scheme, int reach,
                                       const float* d_in, float* d_out, const paraprox_image* img,
                                       const float* d_top, int top_rows, const float* d_bot, int bot_rows,

@@ -506,3 +506,20 @@ def test_concurrent_streams_and_threads(P):
         for (e0, a0, q0, t0), (e1, a1, q1, t1) in zip(seq[k], par[k]):
             assert torch.equal(e0, e1) and torch.equal(a0, a1), k
             assert q0 == q1 and t0 == t1, (k, q0, q1, t0, t1)
+
+
+def test_generic_kernels_tall_images(P, O):
+    """More than 65535 x 8 rows on the fallback kernels (pitch 5 is not
+    TMA-describable): they grid-stride over rows."""
+    x = W.images.random_integers((1, 600001, 5), seed=4, lo=16, hi=235)
+    w = F.mean(5)
+    f = P.Filter(w)
+    for scheme, d in (("exact", 0), ("row", 1)):
+        g = P.stencil_approx(dev(x), f, scheme, d).cpu().numpy()
+        assert P.last_kernel() == "generic", P.last_kernel()
+        o = O.stencil_approx(x, w, scheme, d)
+        assert np.all(np.abs(g - o) <= RTOL * O.stencil_approx(np.abs(x), np.abs(w), scheme, d) + 1e-30), scheme
+    g = P.stencil_lattice(dev(x), f, "col", 1).cpu().numpy()
+    assert P.last_kernel() == "lattice_generic", P.last_kernel()
+    o = O.stencil_lattice(x, w, "col", 1)
+    assert np.all(np.abs(g - o) <= RTOL * O.stencil_lattice(np.abs(x), np.abs(w), "col", 1) + 1e-30)

@@ -155,3 +155,18 @@ def test_hotspot_peer_stripes_ipc(world):
         p.join(timeout=60)
     for r in range(world):
         assert res[r] == "ok", res[r]
+
+
+def test_peer_neighbour_thinner_than_halo_is_refused(P):
+    """A neighbour stripe with fewer rows than the plan's h_y cannot supply the
+    halo (its first row is not the image edge): INVALID_ARG, no launch."""
+    f = mkf(P, F.conv(9))  # exact: h_y = 4
+    x = torch.from_numpy(W.image(40, 64, 6)).cuda()
+    stripe = x[10:30].clone()
+    with pytest.raises(P.ParaproxError):
+        P.stencil_peer(stripe, f, "exact", 0, top=x[8].data_ptr(), top_rows=2, bot=x[30].data_ptr(), bot_rows=4,
+                       src_pitch=x.stride(0))
+    # h_y = 0 (row scheme at full reach): any neighbour is fine, nothing is read
+    got = P.stencil_peer(stripe, f, "row", 4, top=x[8].data_ptr(), top_rows=2, bot=x[30].data_ptr(), bot_rows=1,
+                         src_pitch=x.stride(0))
+    assert torch.equal(got, P.stencil_approx(x, f, "row", 4)[10:30])
