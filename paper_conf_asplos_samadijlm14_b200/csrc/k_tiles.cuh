@@ -390,6 +390,30 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
                 qw[k] = (y < A.h && x0 + wc < A.w) ? __ldcs(rb + (long long)y * A.rpitch) : 0.f;
             }
         }
+        // 3x3 plans with an additive input (HotSpot single steps): the thread's
+        // rows of p are requested before the FMAs, like the Q references
+        constexpr bool ADDPF = !SEP && !Q && HY <= 1 && HX <= 1;
+        float4 pa[ADDPF ? kRB : 1];
+        if constexpr (ADDPF) {
+            if (A.addp) {
+                const float* ab = A.addp + (long long)f * A.afs + x;
+#pragma unroll
+                for (int k = 0; k < kRB; ++k) {
+                    const int y = y0 + ty0 + k;
+                    pa[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (y < A.h && x < A.w) {
+                        const float* ap = ab + (long long)y * A.apitch;
+                        if (x + 3 < A.w) {
+                            pa[k] = __ldcs(reinterpret_cast<const float4*>(ap));
+                        } else {
+                            pa[k].x = ap[0];
+                            if (x + 1 < A.w) pa[k].y = ap[1];
+                            if (x + 2 < A.w) pa[k].z = ap[2];
+                        }
+                    }
+                }
+            }
+        }
         float4 qv[Q && !WIDE ? kRB : 1];  // Q: this thread's reference values, in flight during the FMAs
         if constexpr (Q && !WIDE) {
             const float* rb = A.refp + (long long)f * A.rfs + x;
@@ -682,6 +706,25 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
 #pragma unroll
                 for (int c = 0; c < 4; ++c)
                     if (x + c < A.w) racc.add(A.metric, A.ref_exact ? q4[c] : r4[c], A.ref_exact ? r4[c] : q4[c]);
+            }
+        } else if (ADDPF && A.addp) {
+#pragma unroll
+            for (int k = 0; k < kRB; ++k) {
+                const int y = y0 + ty0 + k;
+                if (y >= A.h || x >= A.w) continue;
+                const float r4[4] = {acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y};
+                const float a4[4] = {pa[k].x, pa[k].y, pa[k].z, pa[k].w};
+                float o4[4];
+#pragma unroll
+                for (int c = 0; c < 4; ++c) o4[c] = __fadd_rn(__fmaf_rn(A.alpha, a4[c], r4[c]), A.beta);
+                float* o = A.out + (long long)f * A.ofs + (long long)y * A.opitch + x;
+                if (x + 3 < A.w) {
+                    __stcs(reinterpret_cast<float4*>(o), make_float4(o4[0], o4[1], o4[2], o4[3]));
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (x + c < A.w) __stcs(o + c, o4[c]);
+                }
             }
         } else if (A.addp) {
             float r[kRB][4];
