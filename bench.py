@@ -451,7 +451,9 @@ def main():
         distinct = [torch.from_numpy(W.image(h, wd, seed_base + 10 + k)).to(dev).view(1, h, wd) for k in range(2)]
         held = distinct
     else:
-        distinct = W.frames(min(n, 16), h, wd, seed_base + 10)
+        # 16 distinct frames over the whole job (c3: 16 x 16 replicas), split
+        # over the ranks so that the host-side generation does not grow with N
+        distinct = W.frames(min(n, max(2, 16 // ws)), h, wd, seed_base + 10)
         t = torch.empty((n, h, wd), device=dev)
         for k in range(n):
             t[k].copy_(torch.from_numpy(distinct[k % len(distinct)]))
