@@ -1,13 +1,13 @@
 #!/bin/bash
-# Multi-GPU runs on one node (needs N GPUs): the default bench (c2, weak),
-# c3 (256 frames split over the ranks, strong) and c4 (row stripes with
-# in-kernel peer halos, strong; --halo nccl for the NCCL exchange).
+# Multi-GPU runs on one node (needs N GPUs): the default bench c3 (256 frames
+# split over the ranks, strong), c2 (weak replicas) and c4 (row stripes,
+# strong; the line times both the in-kernel peer halos and the NCCL exchange).
 # Usage: bash tools/scaling.sh [max_gpus]
 mkdir -p gpurun_out
 MAX=${1:-8}
 for n in 1 2 4 8; do
   [ $n -gt $MAX ] && break
-  for wl in c2 c3 c4; do
+  for wl in c3 c2 c4; do
     if [ $n -eq 1 ]; then
       timeout 900 python bench.py --workload $wl --steps 20 --warmup 3 --no-cpu-baseline > gpurun_out/scale_${wl}_n$n.json 2> gpurun_out/scale_${wl}_n$n.err
     else
