@@ -79,7 +79,7 @@ def hotspot_md(rows, tag):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--round", default="r01")
+    ap.add_argument("--round", default="r02")
     a = ap.parse_args()
     tag = a.round
     for c in ("c1", "c2", "c3", "c4"):
