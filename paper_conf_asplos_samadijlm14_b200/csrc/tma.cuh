@@ -83,7 +83,9 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 // Encodes a 3-D fp32 tensor map [n, rows, w] (strides in elements) with a
 // (box_w, box_h, 1) box.  Returns false if TMA cannot describe the layout
 // (alignment, stride or size limits); callers then use another kernel.
+// l2_promo: bytes an L2 miss of the loads fetches (0, 64, 128, 256; the tile
+// kernels 256: r01 A/B within +-1 %)
 bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n, long long pitch,
-                    long long fstride, int box_w, int box_h);
+                    long long fstride, int box_w, int box_h, int l2_promo = 256);
 
 }  // namespace ppx

@@ -24,10 +24,15 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
 
 // L2 promotion of the TMA loads: 256 B (r01 A/B of none / 64 / 128 / 256 B:
 // within +-1 %)
-static CUtensorMapL2promotion l2_promotion() { return CU_TENSOR_MAP_L2_PROMOTION_L2_256B; }
+static CUtensorMapL2promotion l2_promotion(int bytes) {
+    return bytes >= 256 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B
+                        : bytes >= 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+                                       : bytes >= 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                                                     : CU_TENSOR_MAP_L2_PROMOTION_NONE;
+}
 
 bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n, long long pitch,
-                    long long fstride, int box_w, int box_h) {
+                    long long fstride, int box_w, int box_h, int l2_promo) {
     auto enc = get_encoder();
     if (!enc) return false;
     if ((reinterpret_cast<uintptr_t>(base) & 15) != 0) return false;
@@ -39,7 +44,7 @@ bool encode_tmap_3d(CUtensorMap* map, const float* base, int w, int rows, int n,
     cuuint32_t box[3] = {(cuuint32_t)box_w, (cuuint32_t)box_h, 1};
     cuuint32_t estr[3] = {1, 1, 1};
     CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(base), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, l2_promotion(),
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, l2_promotion(l2_promo),
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
