@@ -27,7 +27,8 @@ timeout 600 python tools/kbench.py --workloads c1,c2,c3,c4 --reps 20 > gpurun_ou
 timeout 600 python tools/convsep.py > gpurun_out/convsep.log 2>&1; echo convsep rc=$?
 timeout 600 python tools/hotspot.py > gpurun_out/hotspot.log 2>&1; echo hotspot rc=$?
 timeout 600 python tools/launch_overhead.py > gpurun_out/launch_overhead.log 2>&1; echo launch-overhead rc=$?
-bash tools/sanitize.sh
+# compute-sanitizer: closed on the GPU pool since the r02 final round (tools/sanitize.sh; r02_sanitizers.md
+# is the last run, all four tools clean)
 # summarise the ncu captures here on the box (gpurun_out/ must stay < 64 MiB)
 if [ -f gpurun_out/prof_c3.ncu-rep ]; then
   python tools/ncu_summary.py full gpurun_out/prof_c3.ncu-rep --workload c3 --traffic gpurun_out/traffic_box.json > gpurun_out/ncu_full_c3.md 2>/dev/null
