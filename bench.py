@@ -388,6 +388,9 @@ def run_stripes(args, dist, rank, ws, local):
             "clocks": clk.summary(), "gpu_launches": launches,
             "e2e": None, "cpu_baseline": None,
         }
+        if ws > torch.cuda.device_count():  # gloo dry run: ranks share one GPU
+            line["ranks_share_device"] = {"ranks": ws, "devices": torch.cuda.device_count(),
+                                          "note": "dry run of the multi-rank path; not a scaling measurement"}
         print(json.dumps(line), flush=True)
     dist.barrier()
     ps.close()
@@ -850,6 +853,12 @@ def main():
             "e2e": e2e,
             "cpu_baseline": cpu,
         }
+        if ws > torch.cuda.device_count():
+            # several ranks on one device (PARAPROX_DIST_BACKEND=gloo dry runs):
+            # the ranks' kernels share one GPU's HBM, so value / hbm_gbs are not
+            # scaling numbers (they can read above the one-GPU peak)
+            line["ranks_share_device"] = {"ranks": ws, "devices": torch.cuda.device_count(),
+                                          "note": "dry run of the multi-rank path; not a scaling measurement"}
         print(json.dumps(line), flush=True)
     if dist:
         dist.barrier()
