@@ -129,7 +129,7 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
     CUtensorMap omap = tmap;  // (unused unless A.tma_store)
     const bool tma_store = !qo && !add && tma_store_enabled() &&
                            encode_tmap_3d(&omap, out, v.w, v.h, v.n, opitch, v.n > 1 ? ofs : (long long)v.h * opitch,
-                                          kTW, e.ti.th);
+                                          kTW, e.ti.store_rows);
     {
         std::lock_guard<std::mutex> lk(g_mu);
         if (!e.ready[dev]) {

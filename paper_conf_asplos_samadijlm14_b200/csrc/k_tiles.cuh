@@ -298,6 +298,17 @@ __host__ __device__ constexpr bool odd_pairs_faster() {
     return HY == 3 && HX == 4 && MASKY == ((1u << 5) | (1u << 8) | (1u << 11)) && MASKX == (0x1FFu << 4);
 }
 
+// FMA-bound plans (the exact 9x9, 81 FMAs per output) store each warp's 8
+// output rows with its own TMA store from a per-warp shared buffer, so the
+// epilogue takes no CTA barrier (the shared-stage epilogue below needs two:
+// the outputs overwrite input rows other warps still read).  r02 ncu of the
+// 9x9: barrier, fence and reconvergence samples 7 % of the kernel's stalls.
+template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
+__host__ __device__ constexpr bool warp_store() {
+    return !SEP && HY == 4 && HX == 4 && MASKY == (0x1FFu << 4) && MASKX == (0x1FFu << 4);
+}
+constexpr int kWarpStoreBytes = kRB * kTW * 4;  // one warp's output rows
+
 template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP, bool Q>
 __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
                                   (tile_min_blocks<HY, HX, MASKY, MASKX, SEP>()))
@@ -370,7 +381,7 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
             const int ahead = tile_at(it + G::STAGES - 1);
             if (in_range(ahead)) {
                 // the stage refilled held the previous tile's output (TMA store)
-                if (A.tma_store) bulk_wait_read_all();
+                if (A.tma_store && !warp_store<HY, HX, MASKY, MASKX, SEP>()) bulk_wait_read_all();
                 issue(ahead, (it + G::STAGES - 1) % G::STAGES);
             }
         }
@@ -737,6 +748,22 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
             }
             tile_epilogue_add(A.addp, A.apitch, A.afs, A.alpha, A.beta, A.out, A.opitch, A.ofs, A.h, A.w, f, y0 + ty0,
                               x, r);
+        } else if (warp_store<HY, HX, MASKY, MASKX, SEP>() && A.tma_store) {
+            // this warp's rows into its own buffer (after its previous TMA
+            // store has read it), one TMA store of kRB x kTW per warp
+            float* O = reinterpret_cast<float*>(smem_raw + G::STAGES * G::STAGE_STRIDE + wi * kWarpStoreBytes);
+            if (lane == 0) bulk_wait_read_all();
+            __syncwarp();
+#pragma unroll
+            for (int k = 0; k < kRB; ++k)
+                reinterpret_cast<float4*>(O + k * kTW)[lane] =
+                    make_float4(acc[k][0].x, acc[k][0].y, acc[k][1].x, acc[k][1].y);
+            fence_proxy_async();  // generic-proxy writes -> visible to the TMA unit
+            __syncwarp();
+            if (lane == 0) {
+                tma_store_3d(&omap, O, x0, y0 + ty0, f);
+                bulk_commit();
+            }
         } else if (A.tma_store) {
             // the tile's outputs replace its consumed input stage ([TH][kTW])
             // and leave as one TMA store (out-of-image elements are clipped)
@@ -771,7 +798,7 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
         }
         __syncthreads();  // stage s fully consumed before it is refilled
     }
-    if (A.tma_store && tid == 0) bulk_wait_all();
+    if (A.tma_store && (warp_store<HY, HX, MASKY, MASKX, SEP>() ? lane == 0 : tid == 0)) bulk_wait_all();
     if constexpr (Q) {  // deterministic: fixed tile order per CTA, fixed reduction tree
         double s0, s1;
         racc.get(A.metric, s0, s1);
@@ -796,6 +823,7 @@ struct TileInstance {
     int smem;
     int threads, th;  // CTA size and tile rows (tile_warps)
     int sw;           // staged row length = the TMA box width (floats)
+    int store_rows;   // rows of one TMA output store (th, or kRB for per-warp stores)
     const char* name;
 };
 
@@ -811,10 +839,12 @@ TileInstance make_instance(const char* name) {
     ti.hx = HX;
     ti.fn = k_tiles<HY, HX, MASKY, MASKX, SEP, false>;
     ti.fnq = k_tiles<HY, HX, MASKY, MASKX, SEP, true>;
-    ti.smem = GeomOf<HY, HX, MASKY, MASKX, SEP>::SMEM;
+    constexpr bool WS = warp_store<HY, HX, MASKY, MASKX, SEP>();
+    ti.smem = GeomOf<HY, HX, MASKY, MASKX, SEP>::SMEM + (WS ? tile_warps<HY, HX, MASKY, MASKX, SEP>() * kWarpStoreBytes : 0);
     ti.threads = 32 * tile_warps<HY, HX, MASKY, MASKX, SEP>();
     ti.th = GeomOf<HY, HX, MASKY, MASKX, SEP>::TH;
     ti.sw = GeomOf<HY, HX, MASKY, MASKX, SEP>::SW;
+    ti.store_rows = WS ? kRB : ti.th;
     ti.name = name;
     return ti;
 }
