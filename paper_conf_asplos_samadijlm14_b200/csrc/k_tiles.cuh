@@ -120,6 +120,9 @@ template <int HY, int HX, uint32_t MASKY, uint32_t MASKX, bool SEP>
 __host__ __device__ constexpr int tile_min_blocks() {
     constexpr uint32_t F2 = 0x1Fu << 6, F4 = 0x1FFu << 4;
     constexpr uint32_t L3 = (1u << 5) | (1u << 8) | (1u << 11), L4 = (1u << 4) | (1u << 8) | (1u << 12);
+    // the wide separable path (sep_wide): 3 CTAs of 8 warps (2 stages of
+    // 37.9 KB; <= 85 registers, the r02 measurement's occupancy)
+    if (SEP && HX > 4) return 3;
     const int b = (!SEP && ((HY == 2 && HX == 2 && MASKY == F2 && MASKX == F2) ||
                             (HY == 3 && HX == 4 && MASKY == L3 && MASKX == F4) ||
                             (HY == 4 && HX == 4 && MASKY == L4 && MASKX == L4)))
@@ -647,6 +650,19 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
                     const float rv = (k & 1) ? vp[k / 2].y : vp[k / 2].x;
                     if (y0 + WR * wh + k < A.h && xo < A.w)
                         racc.add(A.metric, A.ref_exact ? qw[k] : rv, A.ref_exact ? rv : qw[k]);
+                }
+            } else if (A.tma_store) {
+                // outputs replace the consumed stage as a dense [TH][kTW] box,
+                // one TMA store per tile (the register stores below cost ~5
+                // integer instructions per stored float: 64-bit row pointers)
+                __syncthreads();  // every thread has read its staged rows
+#pragma unroll
+                for (int k = 0; k < WR; ++k) S[(WR * wh + k) * kTW + wc] = (k & 1) ? vp[k / 2].y : vp[k / 2].x;
+                fence_proxy_async();
+                __syncthreads();
+                if (tid == 0) {
+                    tma_store_3d(&omap, S, x0, y0, f);
+                    bulk_commit();
                 }
             } else if (xo < A.w) {
                 float* ob = A.out + (long long)f * A.ofs + (long long)(y0 + WR * wh) * A.opitch + xo;
