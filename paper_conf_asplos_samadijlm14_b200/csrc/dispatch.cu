@@ -221,6 +221,13 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
         }
     }
     if (qo) qo->grid = grid;  // one partial pair per CTA, grid <= qo->cap_pairs
+    {  // the stride as (frames, tile rows, tile columns): the kernel's TileWalk
+        const long long tpf = (long long)A.tiles_x * A.tiles_y;
+        A.step_f = (int)(A.stride / tpf);
+        const long long r = A.stride - (long long)A.step_f * tpf;
+        A.step_ty = (int)(r / A.tiles_x);
+        A.step_tx = (int)(r - (long long)A.step_ty * A.tiles_x);
+    }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(e.ti.threads);

@@ -79,6 +79,7 @@ struct LatArgs {
     float* out;
     long long opitch, ofs;
     int stride, chunk;  // tile schedule, as TileArgs (bounded persistence)
+    int step_f, step_ty, step_tx;  // the stride as (frames, tile rows, tile columns): TileWalk
 };
 
 // Row-pair form for the dense s = 3 lattice (the compute-bound one: 27-36
@@ -112,19 +113,13 @@ __global__ void __launch_bounds__(32 * lat_warps<SEP>(), kLatMinBlocks * 8 / lat
     const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
     const int tiles_per_frame = A.tiles_x * A.tiles_y;
 
-    auto coords = [&](int t, int& f, int& y0, int& x0) {
-        f = t / tiles_per_frame;
-        const int r = t - f * tiles_per_frame;
-        const int ty = r / A.tiles_x;
-        y0 = ty * TH;
-        x0 = (r - ty * A.tiles_x) * kTW;
-    };
-    auto issue = [&](int t, int s) {
-        int f, y0, x0;
-        coords(t, f, y0, x0);
+    TileWalk wiss{}, wcur{};  // the issuing thread's walk (tiles ahead), every thread's walk (k_tiles.cuh)
+    auto issue = [&](int s) {  // the tile at wiss
         fence_proxy_async();
         mbar_expect_tx(&bars[s], G::STAGE_BYTES);
-        tma_load_3d(smem_raw + s * G::STAGE_STRIDE, &tmap, x0 - HXP, y0 / S + MLO, f, &bars[s]);
+        tma_load_3d(smem_raw + s * G::STAGE_STRIDE, &tmap, wiss.tx * kTW - HXP, wiss.ty * (TH / S) + MLO, wiss.f,
+                    &bars[s]);
+        wiss.step(A.step_f, A.step_ty, A.step_tx, A.tiles_x, A.tiles_y);
     };
 
     if (tid == 0) {
@@ -140,22 +135,21 @@ __global__ void __launch_bounds__(32 * lat_warps<SEP>(), kLatMinBlocks * 8 / lat
     const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
     const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
                                                : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
+    wcur.init((int)min(t_base, (long long)INT_MAX), A.tiles_x, tiles_per_frame);
+    wiss = wcur;
     if (tid == 0)
-        for (int s = 0; s < G::STAGES - 1; ++s) {
-            const long long t = t_base + (long long)s * A.stride;
-            if (t < t_end) issue((int)t, s);
-        }
+        for (int s = 0; s < G::STAGES - 1; ++s)
+            if (t_base + (long long)s * A.stride < t_end) issue(s);
 
     int it = 0;
     for (long long tl = t_base; tl < t_end; tl += A.stride, ++it) {
-        const int tile = (int)tl;
         const int s = it % G::STAGES;
         if (tid == 0) {
             const long long ahead = tl + (long long)(G::STAGES - 1) * A.stride;
-            if (ahead < t_end) issue((int)ahead, (it + G::STAGES - 1) % G::STAGES);
+            if (ahead < t_end) issue((it + G::STAGES - 1) % G::STAGES);
         }
-        int f, y0, x0;
-        coords(tile, f, y0, x0);
+        const int f = wcur.f, y0 = wcur.ty * TH, x0 = wcur.tx * kTW;
+        wcur.step(A.step_f, A.step_ty, A.step_tx, A.tiles_x, A.tiles_y);
         float* Sm = reinterpret_cast<float*>(smem_raw + s * G::STAGE_STRIDE);
         mbar_wait(&bars[s], (it / G::STAGES) & 1);
 
@@ -490,6 +484,13 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
     long long grid = nt < cap ? nt : cap;
     A.stride = (int)grid;
     A.chunk = lattice_chunk();
+    {
+        const long long tpf = (long long)A.tiles_x * A.tiles_y;
+        A.step_f = (int)(A.stride / tpf);
+        const long long r = A.stride - (long long)A.step_f * tpf;
+        A.step_ty = (int)(r / A.tiles_x);
+        A.step_tx = (int)(r - (long long)A.step_ty * A.tiles_x);
+    }
     if (A.chunk != INT_MAX) {
         const long long waves = (nt + grid * A.chunk - 1) / (grid * A.chunk);
         if (waves * grid >= (1LL << 31)) return launch_lattice_generic(lf, in, v, out, opitch, ofs, dy, dx, s);

@@ -56,6 +56,28 @@ struct TapW {
     float2 wyp[17], wxp[17];
 };
 
+// Tile coordinates along a CTA's walk t_base, t_base + stride, ...: two
+// divisions for the first tile, then the stride's (frames, tile rows, tile
+// columns) decomposition (host-computed) added with carries.  r02 ncu source
+// view: the per-tile divisions were ~70 instructions per warp and a MUFU.RCP
+// latency stall at every tile start (the lattice kernel's top non-FMA stall).
+struct TileWalk {
+    int f, ty, tx;
+    __device__ __forceinline__ void init(int t, int tiles_x, int tpf) {
+        f = t / tpf;
+        const int r = t - f * tpf;
+        ty = r / tiles_x;
+        tx = r - ty * tiles_x;
+    }
+    __device__ __forceinline__ void step(int sf, int sty, int stx, int tiles_x, int tiles_y) {
+        tx += stx;
+        ty += sty;
+        f += sf;
+        if (tx >= tiles_x) tx -= tiles_x, ++ty;
+        if (ty >= tiles_y) ty -= tiles_y, ++f;
+    }
+};
+
 struct TileArgs {
     int n, h, w;
     int rows_valid;  // valid input rows per frame (descriptor rows)
@@ -87,6 +109,7 @@ struct TileArgs {
     // base = (b / stride) * stride * chunk + b % stride (stride = the resident
     // CTAs); chunk = INT_MAX is the fully persistent grid (b + k * gridDim)
     int stride, chunk;
+    int step_f, step_ty, step_tx;  // stride = (step_f * tiles_y + step_ty) * tiles_x + step_tx
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -326,19 +349,14 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
     const int tid = threadIdx.x, lane = tid & 31, wi = tid >> 5;
     const int tiles_per_frame = A.tiles_x * A.tiles_y;
 
-    auto coords = [&](int t, int& f, int& y0, int& x0) {
-        f = t / tiles_per_frame;
-        const int r = t - f * tiles_per_frame;
-        const int ty = r / A.tiles_x;
-        y0 = ty * TH;
-        x0 = (r - ty * A.tiles_x) * kTW;
-    };
-    auto issue = [&](int t, int s) {
-        int f, y0, x0;
-        coords(t, f, y0, x0);
+    // the issuing thread's walk (tiles ahead) and every thread's walk
+    TileWalk wiss{}, wcur{};
+    auto issue = [&](int s) {  // the tile at wiss
         fence_proxy_async();
         mbar_expect_tx(&bars[s], G::STAGE_BYTES);
-        tma_load_3d(smem_raw + s * G::STAGE_STRIDE, &tmap, x0 - HXP, y0 + A.row_off - HY, f, &bars[s]);
+        tma_load_3d(smem_raw + s * G::STAGE_STRIDE, &tmap, wiss.tx * kTW - HXP, wiss.ty * TH + A.row_off - HY, wiss.f,
+                    &bars[s]);
+        wiss.step(A.step_f, A.step_ty, A.step_tx, A.tiles_x, A.tiles_y);
     };
 
     if (tid == 0) {
@@ -370,11 +388,11 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
                                                : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
     auto tile_at = [&](int k) { return (int)min(t_base + (long long)k * A.stride, (long long)INT_MAX); };
     auto in_range = [&](int t) { return t < t_end; };
+    wcur.init(tile_at(0), A.tiles_x, tiles_per_frame);
+    wiss = wcur;
     if (tid == 0)
-        for (int s = 0; s < G::STAGES - 1; ++s) {
-            const int t = tile_at(s);
-            if (in_range(t)) issue(t, s);
-        }
+        for (int s = 0; s < G::STAGES - 1; ++s)
+            if (in_range(tile_at(s))) issue(s);
 
     RAcc racc;  // fused-quality partials (Q)
     int it = 0;
@@ -385,11 +403,11 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
             if (in_range(ahead)) {
                 // the stage refilled held the previous tile's output (TMA store)
                 if (A.tma_store && !warp_store<HY, HX, MASKY, MASKX, SEP>()) bulk_wait_read_all();
-                issue(ahead, (it + G::STAGES - 1) % G::STAGES);
+                issue((it + G::STAGES - 1) % G::STAGES);
             }
         }
-        int f, y0, x0;
-        coords(tile, f, y0, x0);
+        const int f = wcur.f, y0 = wcur.ty * TH, x0 = wcur.tx * kTW;
+        wcur.step(A.step_f, A.step_ty, A.step_tx, A.tiles_x, A.tiles_y);
         const int ty0 = wi * kRB;
         const int x = x0 + 4 * lane;
         constexpr bool WIDE = sep_wide<HX, SEP>();
