@@ -227,6 +227,9 @@ static cudaError_t launch_tiles(Entry& e, const Plan& p, const float* in, const 
         const long long r = A.stride - (long long)A.step_f * tpf;
         A.step_ty = (int)(r / A.tiles_x);
         A.step_tx = (int)(r - (long long)A.step_ty * A.tiles_x);
+        A.dv_stride = make_fastdiv(A.stride);
+        A.dv_tpf = make_fastdiv((int)tpf);
+        A.dv_tx = make_fastdiv(A.tiles_x);
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);

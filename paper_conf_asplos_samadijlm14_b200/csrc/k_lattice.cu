@@ -80,6 +80,7 @@ struct LatArgs {
     long long opitch, ofs;
     int stride, chunk;  // tile schedule, as TileArgs (bounded persistence)
     int step_f, step_ty, step_tx;  // the stride as (frames, tile rows, tile columns): TileWalk
+    FastDiv dv_stride, dv_tpf, dv_tx;  // division by stride, tiles per frame, tiles_x (k_tiles.cuh)
 };
 
 // Row-pair form for the dense s = 3 lattice (the compute-bound one: 27-36
@@ -131,11 +132,11 @@ __global__ void __launch_bounds__(32 * lat_warps<SEP>(), kLatMinBlocks * 8 / lat
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     // CTA b takes tiles t_base + k * stride, k < chunk (k_tiles.cuh)
-    const int wave = (int)blockIdx.x / A.stride;
-    const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
+    const int wave = A.dv_stride.div((int)blockIdx.x);
+    const long long t_base = (long long)wave * A.stride * A.chunk + ((int)blockIdx.x - wave * A.stride);
     const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
                                                : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
-    wcur.init((int)min(t_base, (long long)INT_MAX), A.tiles_x, tiles_per_frame);
+    wcur.init((int)min(t_base, (long long)INT_MAX), A.dv_tpf, tiles_per_frame, A.dv_tx, A.tiles_x);
     wiss = wcur;
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s)
@@ -490,6 +491,9 @@ cudaError_t launch_lattice(const paraprox_filter_s& lf, const float* in, const V
         const long long r = A.stride - (long long)A.step_f * tpf;
         A.step_ty = (int)(r / A.tiles_x);
         A.step_tx = (int)(r - (long long)A.step_ty * A.tiles_x);
+        A.dv_stride = make_fastdiv(A.stride);
+        A.dv_tpf = make_fastdiv((int)tpf);
+        A.dv_tx = make_fastdiv(A.tiles_x);
     }
     if (A.chunk != INT_MAX) {
         const long long waves = (nt + grid * A.chunk - 1) / (grid * A.chunk);

@@ -61,12 +61,32 @@ struct TapW {
 // columns) decomposition (host-computed) added with carries.  r02 ncu source
 // view: the per-tile divisions were ~70 instructions per warp and a MUFU.RCP
 // latency stall at every tile start (the lattice kernel's top non-FMA stall).
+// Division by a launch constant d >= 1 for 0 <= n < 2^31 (Granlund-
+// Montgomery): n / d = umulhi(n, m) >> sh with l = ceil(log2 d),
+// m = ceil(2^(31 + l) / d) < 2^32, sh = l - 1 (exact: the error term
+// n (m d - 2^(31+l)) < 2^31 d <= 2^(31+l)); d == 1 is sh = -1.  Replaces the
+// signed-division sequences (MUFU.RCP + ~30 instructions) at every CTA start.
+struct FastDiv {
+    uint32_t m;
+    int sh;
+    __device__ __forceinline__ int div(int n) const {
+        return sh < 0 ? n : (int)(__umulhi((uint32_t)n, m) >> sh);
+    }
+};
+inline FastDiv make_fastdiv(int d) {
+    if (d <= 1) return FastDiv{0u, -1};
+    int l = 0;
+    while ((1ull << l) < (unsigned long long)d) ++l;
+    const unsigned long long p = 1ull << (31 + l);
+    return FastDiv{(uint32_t)((p + (unsigned long long)d - 1) / (unsigned long long)d), l - 1};
+}
+
 struct TileWalk {
     int f, ty, tx;
-    __device__ __forceinline__ void init(int t, int tiles_x, int tpf) {
-        f = t / tpf;
+    __device__ __forceinline__ void init(int t, const FastDiv& dtpf, int tpf, const FastDiv& dtx, int tiles_x) {
+        f = dtpf.div(t);
         const int r = t - f * tpf;
-        ty = r / tiles_x;
+        ty = dtx.div(r);
         tx = r - ty * tiles_x;
     }
     __device__ __forceinline__ void step(int sf, int sty, int stx, int tiles_x, int tiles_y) {
@@ -110,6 +130,7 @@ struct TileArgs {
     // CTAs); chunk = INT_MAX is the fully persistent grid (b + k * gridDim)
     int stride, chunk;
     int step_f, step_ty, step_tx;  // stride = (step_f * tiles_y + step_ty) * tiles_x + step_tx
+    FastDiv dv_stride, dv_tpf, dv_tx;  // division by stride, tiles per frame, tiles_x
 };
 
 __host__ __device__ constexpr int round4(int v) { return (v + 3) & ~3; }
@@ -382,13 +403,13 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
     // chunks, each CTA takes `chunk` tiles of the stride pattern and retires;
     // the block scheduler starts the next wave's CTAs in order as slots free
     // up, which keeps the window compact.
-    const int wave = (int)blockIdx.x / A.stride;
-    const long long t_base = (long long)wave * A.stride * A.chunk + (int)blockIdx.x % A.stride;
+    const int wave = A.dv_stride.div((int)blockIdx.x);
+    const long long t_base = (long long)wave * A.stride * A.chunk + ((int)blockIdx.x - wave * A.stride);
     const long long t_end = A.chunk == INT_MAX ? (long long)A.ntiles
                                                : min((long long)A.ntiles, (long long)(wave + 1) * A.stride * A.chunk);
     auto tile_at = [&](int k) { return (int)min(t_base + (long long)k * A.stride, (long long)INT_MAX); };
     auto in_range = [&](int t) { return t < t_end; };
-    wcur.init(tile_at(0), A.tiles_x, tiles_per_frame);
+    wcur.init(tile_at(0), A.dv_tpf, tiles_per_frame, A.dv_tx, A.tiles_x);
     wiss = wcur;
     if (tid == 0)
         for (int s = 0; s < G::STAGES - 1; ++s)

@@ -18,6 +18,8 @@ CASES = {
     "c4exact": (1, 16384, 16384, "conv9", 0, 0),
     "c4lat": (1, 16384, 16384, "conv9", "lat", 1),
     "c2exact": (1, 4096, 4096, "mean5", 0, 0),
+    "c3exact": (32, 2160, 3840, "sep7", 0, 0),
+    "c1exact": (110, 512, 512, "gauss3", 0, 0),
     "convsep": (16, 2048, 2048, "sep17", 0, 0),
 }
 
@@ -34,7 +36,8 @@ def run(case):
         wy, wx = F.separable(17, seed_y=17, seed_x=71)
         f = P.Filter(wy=wy, wx=wx)
     else:
-        f = P.Filter(F.named(filt)[1])
+        kind, wts = F.named(filt)
+        f = P.Filter(wy=wts[0], wx=wts[1]) if kind == "sep" else P.Filter(wts)
     nbuf = max(2, int(3 * 126e6 // (8 * n * h * w)) + 1)
     base = torch.from_numpy(W.periodic(h, w, tile=min(4096, h), seed=0) if n == 1 else W.frames(n, h, w, 0)).cuda()
     xs = [base.view(n, h, w).clone() for _ in range(nbuf)]
