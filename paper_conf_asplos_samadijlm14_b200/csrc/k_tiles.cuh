@@ -621,10 +621,10 @@ __global__ void __launch_bounds__(32 * tile_warps<HY, HX, MASKY, MASKX, SEP>(),
             for (int q = 0; q < (SH + 31) / 32; ++q) {
                 const int r = lane + 32 * q;
                 const bool live = r < SH && r >= rlo && r <= rhi;
-                float2 h2[8];
-#pragma unroll
-                for (int j = 0; j < 8; ++j) h2[j] = make_float2(0.f, 0.f);
+                float2 h2[8];  // set (from 0) and used only for live rows
                 if (live) {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) h2[j] = make_float2(0.f, 0.f);
                     float v[NW];
                     const float4* p4 = reinterpret_cast<const float4*>(S + r * SW + cw);
 #pragma unroll
